@@ -1,0 +1,393 @@
+#!/usr/bin/env python
+"""Benchmark of the fused stencil-program hot path on B200 (BASELINE.json metric).
+
+One *step* = one pass of the whole hot path over the program: every fused group of the
+plan (plus periodic ghost fills) in quotient-topological order = one timestep of the
+44-kernel / 31-array weather-shaped program (BASELINE config 3, 512x512x128 fp64).
+
+Printed JSON (rank 0, one line): metric/value = grid-points*steps/s of the fused plan with
+inputs resident in HBM (CUDA events on the launch stream, max over ranks), plus the
+roofline of the dominant group kernel, the oracle's CPU baseline, the end-to-end number
+through kf_run_host (host buffers, copies inside the timed region), the unfused plan's
+speed (speedup vs unfused), the projection, Fusion Efficiency (Eq. 12) and SM clocks.
+
+  python bench.py [--gpus N --steps K --warmup W] [--workload weather|tiny|fig3|stress]
+  python bench.py --impl reference ...     # the oracle on host cores, same metric/config
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+METRIC = "fused-program grid-pts·steps/s"
+UNIT = "grid-pts·steps/s"
+
+
+# ---------------------------------------------------------------- workloads
+def workload(name: str):
+    """(program description, input generator, target kwargs, label)."""
+    from workloads import data, programs
+    if name == "weather":
+        desc = programs.weather(n=(512, 512, 128))
+        return desc, data.weather_inputs, dict(tile=(32, 16, 0)), "weather-44k31a-512x512x128-fp64 (BASELINE config 3)"
+    if name == "weather_small":
+        desc = programs.weather(n=(128, 128, 64))
+        return desc, data.weather_inputs, dict(tile=(32, 16, 0)), "weather-44k31a-128x128x64-fp64"
+    if name == "tiny":
+        desc = programs.tiny()
+        return desc, data.uniform, dict(tile=(32, 16, 0)), "tiny-3k3a-32^3-fp32 (BASELINE config 1)"
+    if name == "fig3":
+        desc = programs.fig3(n=(512, 512, 128))
+        return desc, data.fig3_inputs, dict(tile=(32, 16, 0)), "fig3-6k-512x512x128-fp64"
+    if name == "stress":
+        desc = programs.stress(m=2, n=(768, 768, 768))
+        return desc, data.uniform, dict(tile=(32, 16, 0), max_halo=16), "stress-2fields-L25xL25-768^3-fp64 (config 5)"
+    raise SystemExit(f"unknown workload {name}")
+
+
+def choose_plan(prog, target, which: str):
+    import paper_conf_sc_wahibm14_b200 as kf
+    n = prog.nk
+    if which == "unfused":
+        return list(range(n)), "unfused (singletons)"
+    method = kf.SEARCH_BRUTE if n <= 10 else kf.SEARCH_GREEDY
+    plan, _ = prog.search(method, target)
+    return plan, ("brute-force optimum" if method == kf.SEARCH_BRUTE else "greedy search")
+
+
+# ---------------------------------------------------------------- clocks
+class ClockSampler:
+    FIELDS = "clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown," \
+             "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown," \
+             "clocks_event_reasons.sw_power_cap"
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [p.strip() for p in ln.split(",")]
+            if len(parts) < 7:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                mx = float(parts[1])
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[3:7]):
+                if v.lower() in ("active", "1"):
+                    reasons.add(nm)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"]}
+        sm.sort()
+        return {"sm_mhz": sm[len(sm) // 2], "sm_max_mhz": mx, "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def measured_peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        return None
+
+
+def ncu_traffic(kernel_name: str):
+    """Per-launch DRAM bytes of `kernel_name` from the committed ncu summary, if any."""
+    path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    try:
+        d = json.load(open(path))
+        return d.get(kernel_name)
+    except Exception:
+        return None
+
+
+# ---------------------------------------------------------------- CPU baseline (oracle)
+def cpu_baseline(name: str, budget_s: float = 12.0):
+    """The oracle (numpy, 1 thread) on a bounded sample of the same workload."""
+    from oracle import interp
+    from workloads import programs, data
+    if name.startswith("weather"):
+        desc = programs.weather(n=(96, 96, 128))
+        inp = data.weather_inputs(desc, 3)
+        sample = "weather program on a 96x96x128 sub-grid, 1 step per timing (numpy oracle, unfused)"
+    elif name == "tiny":
+        desc = programs.tiny()
+        inp = data.uniform(desc, 1)
+        sample = "tiny 32^3, 1 step per timing"
+    elif name == "fig3":
+        desc = programs.fig3(n=(128, 128, 128))
+        inp = data.fig3_inputs(desc, 3)
+        sample = "fig3 on 128^3, 1 step"
+    else:
+        desc = programs.stress(m=2, n=(96, 96, 96))
+        inp = data.uniform(desc, 5)
+        sample = "stress 2 fields on 96^3, 1 step"
+    t0 = time.perf_counter()
+    steps = 0
+    while True:
+        inp = interp.run(desc, inp, 1)
+        steps += 1
+        if time.perf_counter() - t0 > budget_s:
+            break
+    dt = time.perf_counter() - t0
+    return {"value": desc.npts * steps / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"{sample}; {steps} step(s) in {dt:.1f} s"}
+
+
+# ---------------------------------------------------------------- GPU timing
+def time_plan(ex, dev, scratch, steps, warmup, stream, profile=False):
+    import torch
+    if profile:
+        ex.set_profiling(True)
+    ex.run(dev, scratch, warmup, stream=stream)
+    torch.cuda.synchronize()
+    if profile:
+        ex.set_profiling(True)    # reset accumulators after warm-up
+    if torch.distributed.is_initialized():
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    ex.run(dev, scratch, steps, stream=stream)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1)
+    gt = None
+    if profile:
+        gt = ex.group_times()
+        ex.set_profiling(False)
+    return ms, gt
+
+
+def max_over_ranks(x: float) -> float:
+    import torch
+    if torch.distributed.is_initialized():
+        t = torch.tensor([x], dtype=torch.float64, device="cuda")
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        return float(t.item())
+    return x
+
+
+def run_kf(args):
+    import numpy as np
+    import torch
+    import paper_conf_sc_wahibm14_b200 as kf
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        torch.cuda.set_device(local)
+        torch.distributed.init_process_group("nccl")
+    else:
+        torch.cuda.set_device(0)
+    desc, gen, tkw, label = workload(args.workload)
+    if args.tile:
+        tkw["tile"] = tuple(int(v) for v in args.tile.split(","))
+    if args.stages:
+        tkw["stages"] = args.stages
+    if args.threads:
+        tkw["threads"] = args.threads
+    target = kf.Target(**tkw)
+    prog = kf.Program(desc)
+    plan, plan_kind = choose_plan(prog, target, args.plan)
+    t0 = time.time()
+    ex = kf.Exec(prog, plan, target)
+    jit_s = time.time() - t0
+    # synthetic inputs of the paper-shaped workload (seed 3 + rank: each rank owns its sub-domain)
+    inputs = gen(desc, 3 + rank)
+    dev = kf.device_arrays(prog, inputs)
+    del inputs
+    sb = ex.scratch_bytes()
+    scratch = torch.empty(sb, dtype=torch.uint8, device="cuda") if sb else None
+    stream = torch.cuda.current_stream()
+    info = ex.info()
+    npts = desc.npts
+
+    with ClockSampler(local) as clk:
+        ms, _ = time_plan(ex, dev, scratch, args.steps, args.warmup, stream)
+    ms = max_over_ranks(ms)
+    clocks = clk.summary()
+    # per-group device times over a second timed region (events on the launch stream)
+    ms_prof, (gms, nlaunch) = time_plan(ex, dev, scratch, args.steps, max(1, args.warmup // 2), stream, profile=True)
+    # unfused plan on the same inputs: speedup vs unfused
+    unf = None
+    if not args.no_unfused and args.plan != "unfused":
+        ex_u = kf.Exec(prog, list(range(prog.nk)), target)
+        sb_u = ex_u.scratch_bytes()
+        scr_u = torch.empty(sb_u, dtype=torch.uint8, device="cuda") if sb_u else None
+        ms_u, _ = time_plan(ex_u, dev, scr_u, args.steps, args.warmup, stream)
+        ms_u = max_over_ranks(ms_u)
+        unf = {"ms_per_step": ms_u / args.steps, "bytes_per_step": ex_u.info().compulsory_bytes_per_step}
+        del ex_u, scr_u
+    # end-to-end through the C ABI with host buffers (copies inside the timed region)
+    e2e = None
+    if not args.no_e2e:
+        host = [t.cpu().pin_memory() for t in dev]
+        ex.run_host([h.data_ptr() for h in host], 1, stream=stream.cuda_stream)   # warm (allocs, first full upload)
+        torch.cuda.synchronize()
+        k = max(1, min(args.steps, 3))
+        t0 = time.perf_counter()
+        h2d = d2h = 0
+        for _ in range(k):
+            a, b = ex.run_host([h.data_ptr() for h in host], 1, stream=stream.cuda_stream)
+            h2d, d2h = a, b
+        dt = time.perf_counter() - t0
+        dt = max_over_ranks(dt)
+        e2e = {"value": world * npts * k / dt, "unit": UNIT, "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+               "steps": k, "timing": "host wall clock around kf_run_host (synchronising), max over ranks"}
+        del host
+
+    bytes_step = info.compulsory_bytes_per_step
+    value = world * npts * args.steps / (ms / 1e3)
+    peaks = measured_peaks()
+    hbm_peak = peaks["hbm_gbs"] if peaks and "hbm_gbs" in peaks else 6650.0
+    peak_src = "MEASURED_PEAKS.json hbm_gbs" if peaks else "B200_PROFILING.md fallback 6.65 TB/s"
+    # dominant kernel = the group with the largest device time
+    g_dom = int(np.argmax(gms))
+    gi = ex.group_info(g_dom)
+    launches_dom = args.steps * info.period // info.period
+    t_launch_ms = gms[g_dom] / args.steps
+    achieved = gi.bytes_per_launch / (t_launch_ms / 1e3) / 1e9
+    roofline = {"bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s", "frac": achieved / hbm_peak,
+                "traffic": ncu_traffic(gi.name), "kernel": gi.name, "peak_source": peak_src,
+                "share_of_step": gms[g_dom] / max(1e-9, sum(gms)),
+                "algorithmic_bytes_per_launch": gi.bytes_per_launch,
+                "per_group_ms_per_step": [g / args.steps for g in gms]}
+    achieved_step = bytes_step / (ms / args.steps / 1e3) / 1e9
+    _, _, t_proj = prog.project(plan, target)
+    res = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "dtype": "f64" if desc.dtype == 1 else "f32", "data": "synthetic (seeded, paper-shaped fields)",
+        "config": {"workload": label, "plan": f"{plan_kind}: {info.n_groups} fused groups of {prog.nk} kernels",
+                   "plan_labels": plan, "tile": list(target.tile), "stages": target.stages,
+                   "threads": target.threads, "l2": "inputs larger than L2 (each array > 126 MB), no flush",
+                   "parallelism": f"replicas x{world}" if world > 1 else "1 GPU",
+                   "graph": True, "jit_s": round(jit_s, 2)},
+        "hbm_gbs_compulsory": achieved_step,
+        "frac_of_measured_copy": achieved_step / hbm_peak,
+        "frac_of_nominal_8TBs": achieved_step / 8000.0,
+        "compulsory_bytes_per_step": bytes_step,
+        "projected_ms_per_step": t_proj * 1e3,
+        "roofline": roofline,
+        "gpu_launches": int(info.launches_per_step * args.steps),
+        "clocks": clocks,
+    }
+    if unf:
+        res["unfused"] = unf
+        res["speedup_vs_unfused"] = unf["ms_per_step"] / (ms / args.steps)
+        traffic_ratio = bytes_step / unf["bytes_per_step"]
+        time_ratio = (ms / args.steps) / unf["ms_per_step"]
+        res["fusion_efficiency"] = traffic_ratio / time_ratio        # Eq. 12
+    if e2e:
+        res["e2e"] = e2e
+    if rank == 0 and not args.no_cpu:
+        res["cpu_baseline"] = cpu_baseline(args.workload)
+    if rank == 0:
+        print(json.dumps(res))
+    if world > 1:
+        torch.distributed.barrier()
+        torch.distributed.destroy_process_group()
+
+
+def run_reference(args):
+    """--impl reference: the oracle as it stands on the host cores (rank 0 only)."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    from oracle import interp
+    from workloads import programs, data
+    desc, gen, tkw, label = workload(args.workload)
+    # bounded sample of the same workload: a sub-grid, one oracle step per timed step
+    if args.workload.startswith("weather"):
+        sub = programs.weather(n=(64, 64, 128))
+        sample = "weather program on a 64x64x128 sub-grid of the 512x512x128 workload, 1 step per timed step"
+    elif args.workload == "tiny":
+        sub = desc
+        sample = "tiny 32^3 (full workload)"
+    elif args.workload == "fig3":
+        sub = programs.fig3(n=(64, 64, 128))
+        sample = "fig3 on a 64x64x128 sub-grid"
+    else:
+        sub = programs.stress(m=2, n=(64, 64, 64))
+        sample = "stress on a 64^3 sub-grid"
+    inp = gen(sub, 3)
+    for _ in range(args.warmup):
+        inp = interp.run(sub, inp, 1)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        inp = interp.run(sub, inp, 1)
+    dt = time.perf_counter() - t0
+    value = sub.npts * args.steps / dt
+    res = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": int(os.environ.get("WORLD_SIZE", "1")),
+           "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3,
+           "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+           "dtype": "f64" if desc.dtype == 1 else "f32", "data": "synthetic", "impl": "reference",
+           "config": {"workload": label},
+           "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+           "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(res))
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="kf", choices=["kf", "reference"])
+    ap.add_argument("--workload", default="weather")
+    ap.add_argument("--plan", default="best", choices=["best", "unfused"])
+    ap.add_argument("--tile", default=None)
+    ap.add_argument("--stages", type=int, default=None)
+    ap.add_argument("--threads", type=int, default=None)
+    ap.add_argument("--no-unfused", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3 and args.impl == "kf":
+        args.warmup = 3
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_kf(args)
+
+
+if __name__ == "__main__":
+    main()

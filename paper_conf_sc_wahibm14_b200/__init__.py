@@ -1,0 +1,9 @@
+"""kf -- B200-native fused stencil-program executor (Wahib & Maruyama, SC'14).
+
+The hot path lives in libkf.so (C ABI, include/kf.h): program/DAG builder, legality,
+projection, plan search, NVRTC-JIT'd sm_100a group kernels and the step runtime.
+This package is only the ctypes binding; it never computes anything itself.
+"""
+from ._abi import KfError, lib  # noqa: F401
+from .api import (SEARCH_AUTO, SEARCH_BRUTE, SEARCH_GREEDY, Exec, Program, Target,  # noqa: F401
+                  device_arrays, flush_l2, host_arrays)

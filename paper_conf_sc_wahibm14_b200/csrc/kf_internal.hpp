@@ -1,0 +1,171 @@
+// Internal data structures of the kf host library (not part of the ABI).
+// Host-side C++: program IR, DAG, lowering, legality, projection, search, codegen.
+// Cites PAPER.md lines as P:n; readings Rn are in DESIGN.md.
+#pragma once
+
+#include <array>
+#include <cstdint>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <set>
+#include <string>
+#include <vector>
+
+#include "kf.h"
+
+namespace kf {
+
+struct Error {
+  kf_status st;
+  std::string msg;
+};
+[[noreturn]] void fail(kf_status st, const std::string& msg);
+void set_error(const std::string& msg);
+
+using Off = std::array<int, 3>;
+
+struct Insn {
+  int op, arg;
+  Off d;
+  double imm;
+};
+struct Stmt {
+  int out;
+  std::vector<Insn> rpn;
+  int depth;
+};
+struct Kernel {
+  std::string name;
+  std::vector<Stmt> stmts;
+  std::map<int, std::vector<Off>> reads;  // array -> sorted distinct offsets (footprint)
+  std::vector<int> writes;                // arrays written (statement order)
+  std::set<int> touched;
+  int depth = 0;                          // deepest RPN stack
+  bool writes_array(int x) const;
+};
+
+// A version of an array inside one step: v = 0 is the value at step start, v >= 1 is
+// produced by the v-th writer in program order.
+struct Ver {
+  int x, v;
+  bool operator<(const Ver& o) const { return x != o.x ? x < o.x : v < o.v; }
+  bool operator==(const Ver& o) const { return x == o.x && v == o.v; }
+};
+
+struct Program {
+  int dtype = 0, es = 4;
+  int64_t n[3] = {0, 0, 0};
+  int ghost[3] = {0, 0, 0};
+  int bc[3] = {0, 0, 0};
+  std::vector<std::string> array_names;
+  std::vector<uint32_t> array_flags;
+  std::vector<Kernel> kernels;
+  int n_params = 0;
+  uint32_t flags = 0;
+
+  // ---- derived (program.cpp)
+  int nk = 0, na = 0;
+  std::vector<std::vector<int>> writers;      // per array, writing kernels ascending
+  std::vector<std::vector<int>> readers;      // per array, reading kernels ascending
+  std::vector<std::map<int, int>> ver_read;   // per kernel: array -> version read
+  std::vector<int> cls;                       // kf_array_class
+  std::vector<char> relaxed, step_live;
+  std::vector<kf_edge> edges;                 // canonical, sorted
+  std::vector<std::vector<uint64_t>> reach;   // bitset rows
+  std::vector<std::vector<char>> share;       // sharing adjacency
+  kf_layout layout{};
+  int64_t npts = 0;
+
+  bool reaches(int a, int b) const { return (reach[a][b >> 6] >> (b & 63)) & 1ull; }
+  int writer_of(int x, int v) const { return writers[x][v - 1]; }
+  int vr(int k, int x) const;                 // version of x current before kernel k
+  int vw(int k, int x) const { return vr(k, x) + 1; }   // version kernel k writes
+  std::vector<int> readers_of_version(int x, int v) const;
+};
+
+void build_program(const kf_program_desc* d, Program& p);   // throws Error
+
+// ---------------------------------------------------------------- plans / lowering
+struct Plan {
+  std::vector<int> label;                 // canonical labels
+  std::vector<std::vector<int>> groups;   // kernels per group, ascending
+  int m = 0;
+};
+Plan make_plan(const Program& p, const int32_t* labels);   // V1 checked by caller
+
+struct Ext {
+  bool alive = false;
+  int elo[3] = {0, 0, 0}, ehi[3] = {0, 0, 0};
+};
+
+// SMEM-resident ring of a version inside a fused group (lowering a3).
+struct Ring {
+  Ver ver;
+  bool live_in = false;   // staged by TMA from HBM; else produced in the group
+  int producer = -1;      // kernel producing it (in-group rings)
+  int blo[3], bhi[3];     // box extents beyond T (xy used for SMEM; z for plane range)
+  int wx, hy, px;         // box width, height, padded row pitch (elements)
+  int plane_bytes;        // roundup(px*hy*es, 128)
+  int slots;              // ring depth
+  int A = 0, B = 0;       // live-in: newest/oldest plane offset needed at iteration t
+  int smem_off = 0;       // byte offset in dynamic SMEM
+};
+
+struct GroupLowering {
+  std::vector<int> kernels;               // program order
+  std::map<int, Ext> ext;                 // per kernel
+  std::map<int, int> delay;               // per alive kernel
+  std::vector<Ver> live_in, live_out;
+  std::set<Ver> live_out_set;
+  std::vector<Ring> rings;
+  int smem = 0, regs = 0, depth = 0;
+  int mbar_off = 0;
+  int tile[3];
+  int stages = 2, threads = 256;
+  int ring_of(const Ver& v) const;        // index in rings or -1
+};
+
+std::vector<Ver> group_live_in(const Program& p, const std::vector<int>& g);
+std::vector<Ver> group_live_out(const Program& p, const std::vector<int>& g);
+GroupLowering lower_group(const Program& p, const std::vector<int>& g, const kf_target& t);
+// Validation; returns code (0 ok) and fills why.
+int validate_plan(const Program& p, const Plan& pl, const kf_target& t, kf_violation* why,
+                  std::vector<GroupLowering>* lowered = nullptr);
+std::vector<int> quotient_order(const Program& p, const Plan& pl);   // empty if cyclic
+int check_kinship(const Program& p, const std::vector<int>& g, int gi, kf_violation* why);
+int check_convex(const Program& p, const std::vector<int>& g, int gi, kf_violation* why);
+int check_hazard(const Program& p, const std::vector<int>& g, const GroupLowering& L, int gi, kf_violation* why);
+int check_halo(const Program& p, const GroupLowering& L, const kf_target& t, int gi, kf_violation* why);
+bool quotient_acyclic(const Program& p, const std::vector<int>& label, int m, int* first_bad);
+void check_target(const kf_target* t);
+uint64_t group_bytes(const Program& p, const std::vector<int>& g, uint64_t* rd, uint64_t* wr);
+
+// ---------------------------------------------------------------- codegen
+struct Codegen {
+  std::string source;
+  std::string name;
+};
+Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid);
+
+}  // namespace kf
+
+struct kf_program {
+  kf::Program p;
+};
+
+#define KF_TRY(...)                                       \
+  try {                                                   \
+    __VA_ARGS__;                                               \
+    return KF_OK;                                         \
+  } catch (const Error& e) {                              \
+    set_error(e.msg);                                     \
+    return e.st;                                          \
+  } catch (const std::bad_alloc&) {                       \
+    set_error("host allocation failed");                  \
+    return KF_E_OOM;                                      \
+  } catch (const std::exception& e) {                     \
+    set_error(std::string("internal error: ") + e.what()); \
+    return KF_E_ARG;                                      \
+  }
+

@@ -1,0 +1,14 @@
+// Host-callable launchers of the ahead-of-time helper kernels (kf_kernels.cu).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace kf {
+struct Geom {
+  int64_t pitch, plane;
+  int xoff, nx, ny, nz, gx, gy, gz;
+};
+cudaError_t launch_fill(int axis, void* base, int es, const Geom& g, cudaStream_t s);
+cudaError_t launch_copy_shell(void* dst, const void* src, int es, const Geom& g, cudaStream_t s);
+cudaError_t launch_flush(void* buf, long long bytes, unsigned v, cudaStream_t s);
+}  // namespace kf

@@ -1,0 +1,508 @@
+// Fusion plans: lowering (a3), legality (a2), projection (a4).
+//
+// Legality follows the constraints of the paper's formulation (Fig. 4, Eq. 1.2-1.7,
+// P:236-272) plus the two readings needed to execute a plan on a GPU: the quotient
+// graph must be acyclic (R4) and no tile may read, outside its own tile, an array the
+// group overwrites in HBM (the SMEM/GMEM incoherence of P:52 and P:107; R7).
+// Extended regions implement the halo layers of complex fusion: producers are
+// recomputed on the Minkowski sum of their consumers' regions and footprints (R8).
+// The projection is the codeless upper bound of P:321 reduced to compulsory bytes over
+// peak bandwidth (Eq. 11's LD/ST counts).
+#include <algorithm>
+#include <climits>
+#include <cstring>
+
+#include "kf_internal.hpp"
+
+namespace kf {
+
+static int64_t rup(int64_t a, int64_t b) { return (a + b - 1) / b * b; }
+
+Plan make_plan(const Program& p, const int32_t* labels) {
+  Plan pl;
+  std::map<int, int> m;
+  pl.label.resize(p.nk);
+  for (int k = 0; k < p.nk; k++) {
+    if (labels[k] < 0) fail(KF_E_ILLEGAL_PLAN, "kernel " + std::to_string(k) + " has a negative group label");
+    auto it = m.find(labels[k]);
+    if (it == m.end()) it = m.emplace(labels[k], int(m.size())).first;
+    pl.label[k] = it->second;
+  }
+  pl.m = int(m.size());
+  pl.groups.assign(pl.m, {});
+  for (int k = 0; k < p.nk; k++) pl.groups[pl.label[k]].push_back(k);
+  return pl;
+}
+
+static bool in_group(const std::vector<int>& g, int k) { return std::binary_search(g.begin(), g.end(), k); }
+
+std::vector<Ver> group_live_in(const Program& p, const std::vector<int>& g) {
+  std::set<Ver> s;
+  for (int k : g)
+    for (auto& [x, _] : p.kernels[k].reads) {
+      int v = p.vr(k, x);
+      if (v == 0 || !in_group(g, p.writer_of(x, v))) s.insert(Ver{x, v});
+    }
+  return std::vector<Ver>(s.begin(), s.end());
+}
+
+std::vector<Ver> group_live_out(const Program& p, const std::vector<int>& g) {
+  std::set<Ver> s;
+  for (int k : g)
+    for (int x : p.kernels[k].writes) {
+      int v = p.vw(k, x);
+      bool outside = false;
+      for (int r : p.readers_of_version(x, v))
+        if (!in_group(g, r)) { outside = true; break; }
+      bool final_live = v == int(p.writers[x].size()) && p.step_live[x];
+      if (outside || final_live) s.insert(Ver{x, v});
+    }
+  return std::vector<Ver>(s.begin(), s.end());
+}
+
+int GroupLowering::ring_of(const Ver& v) const {
+  for (size_t i = 0; i < rings.size(); i++)
+    if (rings[i].ver == v) return int(i);
+  return -1;
+}
+
+GroupLowering lower_group(const Program& p, const std::vector<int>& g, const kf_target& t) {
+  GroupLowering L;
+  L.kernels = g;
+  L.tile[0] = t.tile[0];
+  L.tile[1] = t.tile[1];
+  L.tile[2] = t.tile[2];
+  L.stages = t.stages;
+  L.threads = t.threads;
+  L.live_in = group_live_in(p, g);
+  L.live_out = group_live_out(p, g);
+  L.live_out_set = std::set<Ver>(L.live_out.begin(), L.live_out.end());
+  // ---- extended regions, reverse program order (R8)
+  for (auto it = g.rbegin(); it != g.rend(); ++it) {
+    int k = *it;
+    Ext e;
+    auto merge = [&](const int lo[3], const int hi[3]) {
+      if (!e.alive) {
+        for (int a = 0; a < 3; a++) { e.elo[a] = lo[a]; e.ehi[a] = hi[a]; }
+        e.alive = true;
+      } else {
+        for (int a = 0; a < 3; a++) { e.elo[a] = std::max(e.elo[a], lo[a]); e.ehi[a] = std::max(e.ehi[a], hi[a]); }
+      }
+    };
+    for (int x : p.kernels[k].writes)
+      if (L.live_out_set.count(Ver{x, p.vw(k, x)})) {
+        int z[3] = {0, 0, 0};
+        merge(z, z);
+        break;
+      }
+    for (int c : g) {
+      if (c <= k || !L.ext[c].alive) continue;
+      for (auto& [x, offs] : p.kernels[c].reads) {
+        int v = p.vr(c, x);
+        if (v < 1 || p.writer_of(x, v) != k) continue;
+        int lo[3], hi[3];
+        for (int a = 0; a < 3; a++) {
+          int dmin = INT_MAX, dmax = INT_MIN;
+          for (auto& d : offs) { dmin = std::min(dmin, d[a]); dmax = std::max(dmax, d[a]); }
+          lo[a] = L.ext[c].elo[a] - dmin;
+          hi[a] = L.ext[c].ehi[a] + dmax;
+        }
+        merge(lo, hi);
+      }
+    }
+    L.ext[k] = e;
+  }
+  std::vector<int> alive;
+  for (int k : g)
+    if (L.ext[k].alive) alive.push_back(k);
+  // ---- z delays: a consumer runs behind its in-group producers by their dz reach
+  for (int k : alive) {
+    int dk = 0;
+    for (auto& [x, offs] : p.kernels[k].reads) {
+      int v = p.vr(k, x);
+      if (v < 1) continue;
+      int pr = p.writer_of(x, v);
+      if (!in_group(g, pr) || !L.ext[pr].alive) continue;
+      int mz = INT_MIN;
+      for (auto& d : offs) mz = std::max(mz, d[2]);
+      dk = std::max(dk, L.delay[pr] + mz);
+    }
+    L.delay[k] = dk;
+  }
+  const int es = p.es, TX = t.tile[0], TY = t.tile[1], S = t.stages;
+  auto finish_ring = [&](Ring& r) {
+    r.wx = TX + r.blo[0] + r.bhi[0];
+    r.hy = TY + r.blo[1] + r.bhi[1];
+    r.px = int(rup(r.wx, 16 / es));
+    r.plane_bytes = int(rup(int64_t(r.px) * r.hy * es, 128));
+  };
+  // ---- live-in rings (TMA staged)
+  for (const Ver& lv : L.live_in) {
+    std::vector<int> rd;
+    for (int c : alive)
+      if (p.kernels[c].reads.count(lv.x) && p.vr(c, lv.x) == lv.v) rd.push_back(c);
+    if (rd.empty()) continue;
+    Ring r;
+    r.ver = lv;
+    r.live_in = true;
+    int A = INT_MIN, B = INT_MAX;
+    bool first = true;
+    for (int c : rd) {
+      for (auto& d : p.kernels[c].reads.at(lv.x)) {
+        A = std::max(A, d[2] - L.delay[c]);
+        B = std::min(B, d[2] - L.delay[c]);
+        for (int a = 0; a < 3; a++) {
+          int lo = L.ext[c].elo[a] - d[a], hi = L.ext[c].ehi[a] + d[a];
+          if (first) { r.blo[a] = lo; r.bhi[a] = hi; }
+          else { r.blo[a] = std::max(r.blo[a], lo); r.bhi[a] = std::max(r.bhi[a], hi); }
+        }
+        first = false;
+      }
+    }
+    if (!p.relaxed[lv.x])
+      for (int b : alive)
+        if (p.kernels[b].writes_array(lv.x) && L.live_out_set.count(Ver{lv.x, p.vw(b, lv.x)}))
+          A = std::max(A, -L.delay[b]);
+    r.A = A;
+    r.B = B;
+    r.slots = (A - B + 1) + S - 1;
+    finish_ring(r);
+    L.rings.push_back(r);
+  }
+  // ---- in-group rings (intermediates kept on chip)
+  for (int pk : alive)
+    for (int x : p.kernels[pk].writes) {
+      int v = p.vw(pk, x);
+      int mx = INT_MIN;
+      for (int c : alive)
+        if (p.kernels[c].reads.count(x) && p.vr(c, x) == v)
+          for (auto& d : p.kernels[c].reads.at(x)) mx = std::max(mx, L.delay[c] - d[2]);
+      if (mx == INT_MIN) continue;
+      Ring r;
+      r.ver = Ver{x, v};
+      r.live_in = false;
+      r.producer = pk;
+      for (int a = 0; a < 3; a++) { r.blo[a] = L.ext[pk].elo[a]; r.bhi[a] = L.ext[pk].ehi[a]; }
+      r.slots = mx - L.delay[pk] + 1;
+      finish_ring(r);
+      L.rings.push_back(r);
+    }
+  // ---- SMEM layout and the resource model (R20)
+  int off = 0;
+  for (auto& r : L.rings) {
+    r.smem_off = off;
+    off += r.slots * r.plane_bytes;
+  }
+  L.mbar_off = off;
+  L.smem = off + 8 * S + 128;
+  int depth = 1;
+  for (int k : g) depth = std::max(depth, p.kernels[k].depth);
+  L.depth = depth;
+  L.regs = 32 + 2 * (es / 4) * (depth + 3);
+  return L;
+}
+
+std::vector<int> quotient_order(const Program& p, const Plan& pl) {
+  int m = pl.m;
+  std::vector<std::set<int>> succ(m);
+  std::vector<int> indeg(m, 0);
+  for (auto& e : p.edges) {
+    int a = pl.label[e.src], b = pl.label[e.dst];
+    if (a != b && succ[a].insert(b).second) indeg[b]++;
+  }
+  std::set<int> ready;
+  for (int i = 0; i < m; i++)
+    if (!indeg[i]) ready.insert(i);
+  std::vector<int> order;
+  while (!ready.empty()) {
+    int gq = *ready.begin();
+    ready.erase(ready.begin());
+    order.push_back(gq);
+    for (int h : succ[gq])
+      if (--indeg[h] == 0) ready.insert(h);
+  }
+  if (int(order.size()) != m) order.clear();
+  return order;
+}
+
+static bool nonlocal_read(const Program& p, const GroupLowering& L, int a, int x) {
+  const Ext& e = L.ext.at(a);
+  if (!e.alive) return false;
+  for (auto& d : p.kernels[a].reads.at(x))
+    for (int ax = 0; ax < 3; ax++)
+      if (d[ax] - e.elo[ax] < 0 || e.ehi[ax] + d[ax] > 0) return true;
+  return false;
+}
+
+// ---- per-group checks (each returns a kf_violation_code, filling why on failure)
+int check_kinship(const Program& p, const std::vector<int>& g, int gi, kf_violation* why) {
+  if (p.flags & KF_PROG_NO_KINSHIP) return KF_V_OK;
+  std::set<int> seen{g[0]};
+  std::vector<int> fr{g[0]};
+  while (!fr.empty()) {
+    std::vector<int> nx;
+    for (int u : fr)
+      for (int w : g)
+        if (!seen.count(w) && p.share[u][w]) { seen.insert(w); nx.push_back(w); }
+    fr = nx;
+  }
+  for (int b : g)
+    if (!seen.count(b)) {
+      if (why) *why = kf_violation{KF_V_KINSHIP, gi, g[0], b, -1};
+      return KF_V_KINSHIP;
+    }
+  return KF_V_OK;
+}
+
+int check_convex(const Program& p, const std::vector<int>& g, int gi, kf_violation* why) {
+  for (int c = 0; c < p.nk; c++) {
+    if (in_group(g, c)) continue;
+    int src = -1;
+    for (int a : g)
+      if (p.reaches(a, c)) { src = a; break; }
+    if (src < 0) continue;
+    for (int b : g)
+      if (p.reaches(c, b)) {
+        if (why) *why = kf_violation{KF_V_CONVEX, gi, src, c, -1};
+        return KF_V_CONVEX;
+      }
+  }
+  return KF_V_OK;
+}
+
+int check_hazard(const Program& p, const std::vector<int>& g, const GroupLowering& L, int gi, kf_violation* why) {
+  std::set<Ver> lin(L.live_in.begin(), L.live_in.end());
+  for (int b : g) {
+    std::vector<int> ws = p.kernels[b].writes;
+    std::sort(ws.begin(), ws.end());
+    for (int x : ws) {
+      if (p.relaxed[x] || !L.live_out_set.count(Ver{x, p.vw(b, x)})) continue;
+      for (int a : g) {
+        if (!p.kernels[a].reads.count(x)) continue;
+        if (!lin.count(Ver{x, p.vr(a, x)})) continue;
+        if (nonlocal_read(p, L, a, x)) {
+          if (why) *why = kf_violation{KF_V_HAZARD, gi, a, b, x};
+          return KF_V_HAZARD;
+        }
+      }
+    }
+  }
+  return KF_V_OK;
+}
+
+int check_halo(const Program& p, const GroupLowering& L, const kf_target& t, int gi, kf_violation* why) {
+  for (const auto& r : L.rings) {   // live-in rings come first, sorted by (array, version)
+    if (!r.live_in) continue;
+    for (int a = 0; a < 3; a++) {
+      bool wrap = p.bc[a] == KF_BC_PERIODIC || ((t.internal_axes >> a) & 1);
+      int ext = std::max(r.blo[a], r.bhi[a]);
+      if ((wrap && ext > p.ghost[a]) || (a < 2 && ext > t.max_halo)) {
+        if (why) *why = kf_violation{KF_V_HALO, gi, -1, -1, r.ver.x};
+        return KF_V_HALO;
+      }
+    }
+  }
+  for (int k : L.kernels) {
+    const Ext& e = L.ext.at(k);
+    if (!e.alive) continue;
+    if (std::max({e.elo[0], e.ehi[0], e.elo[1], e.ehi[1]}) > t.max_halo) {
+      if (why) *why = kf_violation{KF_V_HALO, gi, k, -1, -1};
+      return KF_V_HALO;
+    }
+  }
+  return KF_V_OK;
+}
+
+bool quotient_acyclic(const Program& p, const std::vector<int>& label, int m, int* first_bad) {
+  std::vector<std::vector<char>> q(m, std::vector<char>(m, 0));
+  for (auto& e : p.edges) {
+    int a = label[e.src], b = label[e.dst];
+    if (a != b) q[a][b] = 1;
+  }
+  for (int k = 0; k < m; k++)
+    for (int i = 0; i < m; i++)
+      if (q[i][k])
+        for (int j = 0; j < m; j++)
+          if (q[k][j]) q[i][j] = 1;
+  for (int gi = 0; gi < m; gi++)
+    if (q[gi][gi]) {
+      if (first_bad) *first_bad = gi;
+      return false;
+    }
+  return true;
+}
+
+int validate_plan(const Program& p, const Plan& pl, const kf_target& t, kf_violation* why,
+                  std::vector<GroupLowering>* lowered) {
+  if (why) *why = kf_violation{KF_V_OK, -1, -1, -1, -1};
+  int c;
+  for (int gi = 0; gi < pl.m; gi++)
+    if ((c = check_kinship(p, pl.groups[gi], gi, why))) return c;
+  for (int gi = 0; gi < pl.m; gi++)
+    if ((c = check_convex(p, pl.groups[gi], gi, why))) return c;
+  int bad = -1;
+  if (!quotient_acyclic(p, pl.label, pl.m, &bad)) {
+    if (why) *why = kf_violation{KF_V_CYCLE, bad, -1, -1, -1};
+    return KF_V_CYCLE;
+  }
+  std::vector<GroupLowering> Ls;
+  for (int gi = 0; gi < pl.m; gi++) Ls.push_back(lower_group(p, pl.groups[gi], t));
+  for (int gi = 0; gi < pl.m; gi++)
+    if ((c = check_hazard(p, pl.groups[gi], Ls[gi], gi, why))) return c;
+  for (int gi = 0; gi < pl.m; gi++)
+    if ((c = check_halo(p, Ls[gi], t, gi, why))) return c;
+  for (int gi = 0; gi < pl.m; gi++)
+    if (Ls[gi].smem > t.smem_per_block) {
+      if (why) *why = kf_violation{KF_V_SMEM, gi, -1, -1, -1};
+      return KF_V_SMEM;
+    }
+  for (int gi = 0; gi < pl.m; gi++)
+    if (Ls[gi].regs > t.regs_per_thread_max) {
+      if (why) *why = kf_violation{KF_V_REGS, gi, -1, -1, -1};
+      return KF_V_REGS;
+    }
+  if (lowered) *lowered = std::move(Ls);
+  return KF_V_OK;
+}
+
+uint64_t group_bytes(const Program& p, const std::vector<int>& g, uint64_t* rd, uint64_t* wr) {
+  uint64_t unit = uint64_t(p.npts) * uint64_t(p.es);
+  uint64_t r = unit * group_live_in(p, g).size();
+  uint64_t w = unit * group_live_out(p, g).size();
+  if (rd) *rd = r;
+  if (wr) *wr = w;
+  return r + w;
+}
+
+void check_target(const kf_target* t) {
+  if (!t) fail(KF_E_ARG, "null target");
+  if (t->tile[0] < 1 || t->tile[1] < 1 || t->tile[2] < 0 || t->tile[0] > 224 || t->tile[1] > 224)
+    fail(KF_E_ARG, "tile must be TX,TY in [1,224], TZ >= 0");
+  if (t->max_halo < 0 || t->max_halo > 16) fail(KF_E_ARG, "max_halo must be in [0,16] (TMA box <= 256)");
+  if (t->stages < 2 || t->stages > 8) fail(KF_E_ARG, "stages must be in [2, 8]");
+  if (t->threads < 32 || t->threads > 1024 || t->threads % 32) fail(KF_E_ARG, "threads must be a multiple of 32 in [32,1024]");
+  if (!(t->hbm_bytes_per_s > 0)) fail(KF_E_ARG, "hbm_bytes_per_s must be > 0");
+}
+
+}  // namespace kf
+
+using namespace kf;
+
+extern "C" {
+
+kf_status kf_plan_canonical(const int32_t* plan, int32_t n, int32_t* out, int32_t* m) {
+  KF_TRY({
+    if (!plan || !out || n < 0) fail(KF_E_ARG, "null argument");
+    std::map<int, int> mp;
+    std::vector<int32_t> r(n);
+    for (int i = 0; i < n; i++) {
+      if (plan[i] < 0) fail(KF_E_ILLEGAL_PLAN, "negative label");
+      auto it = mp.find(plan[i]);
+      if (it == mp.end()) it = mp.emplace(plan[i], int(mp.size())).first;
+      r[i] = it->second;
+    }
+    std::copy(r.begin(), r.end(), out);
+    if (m) *m = int(mp.size());
+  });
+}
+
+kf_status kf_plan_validate(const kf_program* prog, const int32_t* plan, const kf_target* target, kf_violation* why) {
+  try {
+    if (!prog || !plan) fail(KF_E_ARG, "null argument");
+    check_target(target);
+    const Program& p = prog->p;
+    for (int k = 0; k < p.nk; k++)
+      if (plan[k] < 0) {
+        if (why) *why = kf_violation{KF_V_PARTITION, -1, k, -1, -1};
+        set_error("V1 PARTITION: kernel " + std::to_string(k) + " has no group");
+        return KF_E_ILLEGAL_PLAN;
+      }
+    Plan pl = make_plan(p, plan);
+    kf_violation w{};
+    int code = validate_plan(p, pl, *target, &w);
+    if (why) *why = w;
+    if (code != KF_V_OK) {
+      static const char* names[] = {"OK", "V1 PARTITION", "V2 KINSHIP", "V3 CONVEX", "V4 CYCLE",
+                                    "V5 HAZARD", "V6 HALO", "V7 SMEM", "V8 REGS"};
+      set_error(std::string(names[code]) + " in group " + std::to_string(w.group));
+      return KF_E_ILLEGAL_PLAN;
+    }
+    return KF_OK;
+  } catch (const Error& e) {
+    set_error(e.msg);
+    return e.st;
+  } catch (const std::exception& e) {
+    set_error(e.what());
+    return KF_E_ARG;
+  }
+}
+
+kf_status kf_project(const kf_program* prog, const int32_t* plan, const kf_target* target, kf_group_proj* per_group,
+                     int32_t cap, int32_t* m, uint64_t* bytes_total, double* t_total_s) {
+  KF_TRY({
+    if (!prog || !plan) fail(KF_E_ARG, "null argument");
+    check_target(target);
+    const Program& p = prog->p;
+    Plan pl = make_plan(p, plan);
+    if (cap > 0 && !per_group) fail(KF_E_ARG, "per_group is NULL");
+    uint64_t tot = 0;
+    double tt = 0.0;
+    std::vector<kf_group_proj> res;
+    for (int gi = 0; gi < pl.m; gi++) {
+      const auto& g = pl.groups[gi];
+      kf_group_proj r{};
+      group_bytes(p, g, &r.bytes_read, &r.bytes_written);
+      GroupLowering L = lower_group(p, g, *target);
+      r.smem_bytes = uint32_t(L.smem);
+      r.regs_est = uint32_t(L.regs);
+      r.n_kernels = int(g.size());
+      uint64_t unit = uint64_t(p.npts) * p.es;
+      double halo = 0.0;
+      for (auto& rg : L.rings)
+        if (rg.live_in)
+          halo += double(unit) * (double(rg.wx) * rg.hy / (double(L.tile[0]) * L.tile[1]) - 1.0);
+      r.halo_bytes_est = uint64_t(std::max(0.0, halo));
+      if (g.size() >= 2) {
+        uint64_t alone = 0;
+        for (int k : g) alone += group_bytes(p, std::vector<int>{k}, nullptr, nullptr);
+        r.unprofitable = (r.bytes_read + r.bytes_written) >= alone;
+      }
+      r.t_s = double(r.bytes_read + r.bytes_written) / target->hbm_bytes_per_s;
+      tot += r.bytes_read + r.bytes_written;
+      tt += r.t_s;
+      res.push_back(r);
+    }
+    for (int i = 0; i < int(res.size()) && i < cap; i++) per_group[i] = res[i];
+    if (m) *m = pl.m;
+    if (bytes_total) *bytes_total = tot;
+    if (t_total_s) *t_total_s = tt;
+  });
+}
+
+kf_status kf_group_schedule(const kf_program* prog, const int32_t* plan, const kf_target* target, int32_t group,
+                            kf_kernel_sched* out, int32_t cap, int32_t* n) {
+  KF_TRY({
+    if (!prog || !plan || !n) fail(KF_E_ARG, "null argument");
+    check_target(target);
+    const Program& p = prog->p;
+    Plan pl = make_plan(p, plan);
+    if (group < 0 || group >= pl.m) fail(KF_E_ARG, "group out of range");
+    GroupLowering L = lower_group(p, pl.groups[group], *target);
+    int i = 0;
+    for (int k : L.kernels) {
+      if (i < cap && out) {
+        kf_kernel_sched s{};
+        const Ext& e = L.ext.at(k);
+        s.kernel = k;
+        s.alive = e.alive;
+        s.delay = e.alive ? L.delay.at(k) : -1;
+        for (int a = 0; a < 3; a++) { s.elo[a] = e.elo[a]; s.ehi[a] = e.ehi[a]; }
+        out[i] = s;
+      }
+      i++;
+    }
+    *n = i;
+  });
+}
+
+}  // extern "C"

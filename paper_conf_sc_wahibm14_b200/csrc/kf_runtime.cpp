@@ -1,0 +1,710 @@
+// Runtime executor (rows a6, a10): NVRTC JIT of the generated group kernels for sm_100a,
+// module/tensor-map management, renamed-buffer ping-pong, periodic ghost fills, and the
+// step loop (a CUDA graph of one replay period).
+//
+// Host -> device boundary: one graph launch per period; everything inside the step runs
+// in this library's kernels (JIT'd group kernels + AOT helpers in kf_kernels.cu).
+// The paper fused kernels by hand and replaced the calls "from the host by a
+// single call to the newly constructed kernel" (P:39(c)); here the host issues groups in
+// quotient-topological order (R18).
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <nvrtc.h>
+
+#include <algorithm>
+#include <cstring>
+#include <functional>
+#include <sstream>
+
+#include "kf_internal.hpp"
+#include "kf_kernels.hpp"
+
+namespace kf {
+
+// ---------------------------------------------------------------- driver entry points
+struct Drv {
+  CUresult (*moduleLoadData)(CUmodule*, const void*) = nullptr;
+  CUresult (*moduleGetFunction)(CUfunction*, CUmodule, const char*) = nullptr;
+  CUresult (*funcSetAttribute)(CUfunction, CUfunction_attribute, int) = nullptr;
+  CUresult (*funcGetAttribute)(int*, CUfunction_attribute, CUfunction) = nullptr;
+  CUresult (*launchKernel)(CUfunction, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned, CUstream,
+                           void**, void**) = nullptr;
+  CUresult (*tensorMapEncodeTiled)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                   const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                   CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill) = nullptr;
+  CUresult (*getErrorString)(CUresult, const char**) = nullptr;
+};
+
+#define CK(x)                                                                                       \
+  do {                                                                                              \
+    cudaError_t e_ = (x);                                                                           \
+    if (e_ != cudaSuccess) fail(KF_E_CUDA, std::string(#x) + ": " + cudaGetErrorString(e_));        \
+  } while (0)
+
+static Drv& drv() {
+  static Drv d;
+  static std::once_flag once;
+  static std::string err;
+  std::call_once(once, [] {
+    auto get = [](const char* sym, void** fp) {
+      cudaDriverEntryPointQueryResult q;
+      cudaError_t e = cudaGetDriverEntryPoint(sym, fp, cudaEnableDefault, &q);
+      if (e != cudaSuccess || q != cudaDriverEntryPointSuccess) *fp = nullptr;
+    };
+    get("cuModuleLoadData", (void**)&d.moduleLoadData);
+    get("cuModuleGetFunction", (void**)&d.moduleGetFunction);
+    get("cuFuncSetAttribute", (void**)&d.funcSetAttribute);
+    get("cuFuncGetAttribute", (void**)&d.funcGetAttribute);
+    get("cuLaunchKernel", (void**)&d.launchKernel);
+    get("cuTensorMapEncodeTiled", (void**)&d.tensorMapEncodeTiled);
+    get("cuGetErrorString", (void**)&d.getErrorString);
+  });
+  if (!d.moduleLoadData || !d.launchKernel || !d.tensorMapEncodeTiled)
+    fail(KF_E_UNSUPPORTED, "CUDA driver entry points unavailable (no GPU / driver?)");
+  return d;
+}
+
+static void ckd(CUresult r, const char* what) {
+  if (r == CUDA_SUCCESS) return;
+  const char* s = nullptr;
+  if (drv().getErrorString) drv().getErrorString(r, &s);
+  fail(KF_E_CUDA, std::string(what) + ": " + (s ? s : "CUDA driver error " + std::to_string(int(r))));
+}
+
+// ---------------------------------------------------------------- NVRTC
+struct Compiled {
+  std::vector<char> cubin;
+  std::string log;
+  int regs_ptxas = -1, spill = -1;
+};
+
+static Compiled nvrtc_compile(const std::string& src, const std::string& name) {
+  nvrtcProgram prog;
+  if (nvrtcCreateProgram(&prog, src.c_str(), (name + ".cu").c_str(), 0, nullptr, nullptr) != NVRTC_SUCCESS)
+    fail(KF_E_NVRTC, "nvrtcCreateProgram failed");
+  // IEEE semantics, no FMA contraction (R16): fused results must equal the unfused program bit for bit.
+  const char* opts[] = {"--gpu-architecture=sm_100a", "--fmad=false", "--prec-div=true", "--prec-sqrt=true",
+                        "--ftz=false", "-std=c++17", "-lineinfo", "--ptxas-options=-v"};
+  if (getenv("KF_DEBUG")) fprintf(stderr, "nvrtc: compiling %s\n", name.c_str());
+  nvrtcResult r = nvrtcCompileProgram(prog, int(sizeof(opts) / sizeof(opts[0])), opts);
+  if (getenv("KF_DEBUG")) fprintf(stderr, "nvrtc: done %d\n", int(r));
+  Compiled c;
+  size_t ls = 0;
+  nvrtcGetProgramLogSize(prog, &ls);
+  c.log.resize(ls);
+  if (ls) nvrtcGetProgramLog(prog, &c.log[0]);
+  if (r != NVRTC_SUCCESS) {
+    nvrtcDestroyProgram(&prog);
+    fail(KF_E_NVRTC, "NVRTC failed for " + name + ": " + c.log.substr(0, 4000));
+  }
+  size_t cs = 0;
+  nvrtcGetCUBINSize(prog, &cs);
+  c.cubin.resize(cs);
+  nvrtcGetCUBIN(prog, c.cubin.data());
+  nvrtcDestroyProgram(&prog);
+  auto p = c.log.find("Used ");
+  if (p != std::string::npos) c.regs_ptxas = atoi(c.log.c_str() + p + 5);
+  auto q = c.log.find("bytes spill stores");
+  if (q != std::string::npos) {
+    size_t b = c.log.rfind(',', q);
+    b = b == std::string::npos ? 0 : b + 1;
+    c.spill = atoi(c.log.c_str() + b);
+  }
+  return c;
+}
+
+static std::mutex g_cache_mu;
+static std::map<std::string, std::shared_ptr<Compiled>> g_cubin_cache;   // source -> cubin
+
+static std::shared_ptr<Compiled> compile_cached(const std::string& src, const std::string& name) {
+  {
+    std::lock_guard<std::mutex> lk(g_cache_mu);
+    auto it = g_cubin_cache.find(src);
+    if (it != g_cubin_cache.end()) return it->second;
+  }
+  auto c = std::make_shared<Compiled>(nvrtc_compile(src, name));
+  std::lock_guard<std::mutex> lk(g_cache_mu);
+  g_cubin_cache[src] = c;
+  return c;
+}
+
+// ---------------------------------------------------------------- executor
+struct Op {
+  int kind;   // 0 = periodic fill of a buffer, 1 = group launch
+  int group;
+  int buf;
+};
+
+struct GroupExec {
+  int gid = 0;
+  GroupLowering L;
+  Codegen cg;
+  std::shared_ptr<Compiled> comp;
+  CUmodule mod = nullptr;
+  CUfunction fn = nullptr;
+  int grid = 0, smem = 0, regs = -1, local = -1;
+  uint64_t bytes = 0;
+  std::vector<Ver> ins, outs, mids;
+  size_t blob_size = 0;
+};
+
+}  // namespace kf
+
+using namespace kf;
+
+struct kf_exec {
+  kf_program* prog = nullptr;
+  Plan plan;
+  kf_target t{};
+  std::vector<int> order;
+  std::vector<GroupExec> G;
+  int period = 1;
+  std::vector<std::vector<Op>> sched;      // per parity
+  std::vector<Ver> scratch_vers;           // scratch buffer i holds (x, v)
+  uint64_t scratch_bytes = 0, array_bytes = 0;
+  std::vector<int> fill_all;               // buffers filled once at the start of a run
+  int device = -1;
+  // current pointers / argument blobs
+  std::vector<void*> cur_arrays;
+  void* cur_scratch = nullptr;
+  std::vector<double> cur_params;
+  std::vector<std::vector<std::vector<unsigned char>>> blobs;   // [parity][group]
+  bool blobs_valid = false;
+  void* shell_init_scratch = nullptr;
+  std::vector<void*> shell_init_arrays;
+  // graph
+  bool use_graph = true;
+  cudaStream_t cap_stream = nullptr;
+  cudaGraphExec_t gexec = nullptr;
+  // profiling
+  bool profiling = false;
+  std::vector<double> gms;
+  int64_t launches = 0;
+  std::vector<std::tuple<int, cudaEvent_t, cudaEvent_t>> pending;
+  std::vector<cudaEvent_t> evpool;
+  // host-buffer runs
+  std::vector<void*> dev_arrays;
+  void* dev_scratch = nullptr;
+  bool host_first = true;
+  uint64_t step_bytes = 0;
+};
+
+namespace kf {
+
+static int buffer_id(const kf_exec* E, const Ver& v, int parity) {
+  const Program& p = E->prog->p;
+  int x = v.x;
+  if (!p.relaxed[x]) return x;
+  int w = int(p.writers[x].size());
+  auto scr = [&](int ver) {
+    for (size_t i = 0; i < E->scratch_vers.size(); i++)
+      if (E->scratch_vers[i] == Ver{x, ver}) return p.na + int(i);
+    fail(KF_E_ARG, "internal: missing scratch buffer");
+  };
+  if (!p.step_live[x]) {
+    if (v.v == 0 || v.v == w) return x;
+    return scr(v.v);
+  }
+  if (v.v == 0) return parity == 0 ? x : scr(w);
+  if (v.v == w) return parity == 0 ? scr(w) : x;
+  return scr(v.v);
+}
+
+static Geom geom(const Program& p) {
+  Geom g;
+  g.pitch = p.layout.pitch;
+  g.plane = p.layout.plane;
+  g.xoff = p.layout.xoff;
+  g.nx = int(p.n[0]); g.ny = int(p.n[1]); g.nz = int(p.n[2]);
+  g.gx = p.ghost[0]; g.gy = p.ghost[1]; g.gz = p.ghost[2];
+  return g;
+}
+
+static void* buf_ptr(const kf_exec* E, int id) {
+  const Program& p = E->prog->p;
+  if (id < p.na) return E->cur_arrays[id];
+  return (char*)E->cur_scratch + uint64_t(id - p.na) * E->array_bytes;
+}
+
+static void build_blobs(kf_exec* E) {
+  const Program& p = E->prog->p;
+  const int es = p.es;
+  E->blobs.assign(E->period, std::vector<std::vector<unsigned char>>(E->G.size()));
+  for (int par = 0; par < E->period; par++)
+    for (auto& g : E->G) {
+      size_t ni = std::max<size_t>(1, g.ins.size()), no = std::max<size_t>(1, g.outs.size()),
+             nm = std::max<size_t>(1, g.mids.size()), np = std::max(1, p.n_params);
+      size_t sz = 128 * ni + 8 * (no + nm + np);
+      sz = (sz + 63) / 64 * 64;
+      g.blob_size = sz;
+      std::vector<unsigned char> b(sz + 64, 0);
+      // keep 64-byte alignment of the tensor maps inside the blob
+      unsigned char* base = b.data() + ((64 - (reinterpret_cast<uintptr_t>(b.data()) & 63)) & 63);
+      for (size_t i = 0; i < g.ins.size(); i++) {
+        const Ring& R = g.L.rings[g.L.ring_of(g.ins[i])];
+        void* ptr = buf_ptr(E, buffer_id(E, g.ins[i], par));
+        cuuint64_t dims[3] = {cuuint64_t(p.layout.pitch), cuuint64_t(p.layout.rows), cuuint64_t(p.n[2] + 2 * p.ghost[2])};
+        cuuint64_t strides[2] = {cuuint64_t(p.layout.pitch * es), cuuint64_t(p.layout.plane * es)};
+        cuuint32_t box[3] = {cuuint32_t(R.px), cuuint32_t(R.hy), 1};
+        cuuint32_t estr[3] = {1, 1, 1};
+        CUtensorMap* tm = reinterpret_cast<CUtensorMap*>(base + 128 * i);
+        ckd(drv().tensorMapEncodeTiled(tm, es == 4 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3,
+                                       ptr, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                                       CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                                       CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE),
+            "cuTensorMapEncodeTiled");
+      }
+      unsigned char* q = base + 128 * ni;
+      for (size_t j = 0; j < no; j++) {
+        void* ptr = j < g.outs.size() ? (char*)buf_ptr(E, buffer_id(E, g.outs[j], par)) + p.layout.origin * es : nullptr;
+        std::memcpy(q + 8 * j, &ptr, 8);
+      }
+      q += 8 * no;
+      for (size_t j = 0; j < nm; j++) {
+        void* ptr = j < g.mids.size() ? (char*)buf_ptr(E, buffer_id(E, g.mids[j], par)) + p.layout.origin * es : nullptr;
+        std::memcpy(q + 8 * j, &ptr, 8);
+      }
+      q += 8 * nm;
+      for (int j = 0; j < p.n_params; j++) std::memcpy(q + 8 * j, &E->cur_params[j], 8);
+      std::vector<unsigned char> out(base, base + sz);
+      E->blobs[par][&g - &E->G[0]] = std::move(out);
+    }
+  E->blobs_valid = true;
+}
+
+static void launch_group(kf_exec* E, int gi, int par, cudaStream_t s) {
+  GroupExec& g = E->G[gi];
+  std::vector<unsigned char>& blob = E->blobs[par][gi];
+  // The argument block is one __grid_constant__ struct; the driver copies it at launch.
+  alignas(64) unsigned char tmp[32768];
+  if (blob.size() > sizeof(tmp)) fail(KF_E_RESOURCE, "kernel argument block too large");
+  std::memcpy(tmp, blob.data(), blob.size());
+  void* params[] = {tmp};
+  ckd(drv().launchKernel(g.fn, g.grid, 1, 1, g.L.threads, 1, 1, g.smem, (CUstream)s, params, nullptr),
+      ("cuLaunchKernel " + g.cg.name).c_str());
+}
+
+static void run_fill(kf_exec* E, int buf, cudaStream_t s) {
+  const Program& p = E->prog->p;
+  Geom gm = geom(p);
+  for (int a = 0; a < 3; a++)
+    if (p.bc[a] == KF_BC_PERIODIC) CK(launch_fill(a, buf_ptr(E, buf), p.es, gm, s));
+}
+
+static void run_step(kf_exec* E, int par, cudaStream_t s) {
+  for (const Op& op : E->sched[par]) {
+    if (op.kind == 0) {
+      run_fill(E, op.buf, s);
+    } else if (E->profiling) {
+      cudaEvent_t a, b;
+      if (E->evpool.size() >= 2) {
+        a = E->evpool.back(); E->evpool.pop_back();
+        b = E->evpool.back(); E->evpool.pop_back();
+      } else {
+        CK(cudaEventCreate(&a));
+        CK(cudaEventCreate(&b));
+      }
+      CK(cudaEventRecord(a, s));
+      launch_group(E, op.group, par, s);
+      CK(cudaEventRecord(b, s));
+      E->pending.emplace_back(op.group, a, b);
+      E->launches++;
+    } else {
+      launch_group(E, op.group, par, s);
+    }
+  }
+}
+
+static void ensure_device(kf_exec* E) {
+  int dev = 0;
+  CK(cudaGetDevice(&dev));
+  if (E->device >= 0 && dev != E->device) fail(KF_E_ARG, "kf_exec used on a different device than it was created on");
+  if (E->device >= 0) return;
+  CK(cudaFree(nullptr));   // make the primary context current
+  E->device = dev;
+  const Program& p = E->prog->p;
+  for (auto& g : E->G) {
+    ckd(drv().moduleLoadData(&g.mod, g.comp->cubin.data()), ("cuModuleLoadData " + g.cg.name).c_str());
+    ckd(drv().moduleGetFunction(&g.fn, g.mod, g.cg.name.c_str()), "cuModuleGetFunction");
+    ckd(drv().funcSetAttribute(g.fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, g.smem),
+        "cuFuncSetAttribute(MAX_DYNAMIC_SHARED_SIZE_BYTES)");
+    drv().funcGetAttribute(&g.regs, CU_FUNC_ATTRIBUTE_NUM_REGS, g.fn);
+    drv().funcGetAttribute(&g.local, CU_FUNC_ATTRIBUTE_LOCAL_SIZE_BYTES, g.fn);
+  }
+  (void)p;
+}
+
+static void build_schedule(kf_exec* E) {
+  const Program& p = E->prog->p;
+  // periodic-fill needs: live-in rings whose box reaches beyond T on a periodic axis
+  auto needs_fill = [&](const GroupExec& g, const Ver& v) {
+    const Ring& R = g.L.rings[g.L.ring_of(v)];
+    for (int a = 0; a < 3; a++)
+      if (p.bc[a] == KF_BC_PERIODIC && std::max(R.blo[a], R.bhi[a]) > 0) return true;
+    return false;
+  };
+  std::set<int> all_fill;
+  std::vector<std::vector<Op>> sched(E->period);
+  std::set<int> dirty;
+  for (int pass = 0; pass < 2; pass++)
+    for (int par = 0; par < E->period; par++) {
+      std::vector<Op> ops;
+      for (int gi : E->order) {
+        const GroupExec& g = E->G[gi];
+        std::set<int> filled;
+        for (const Ver& v : g.ins) {
+          if (!needs_fill(g, v)) continue;
+          int b = buffer_id(E, v, par);
+          all_fill.insert(b);
+          if (dirty.count(b) && !filled.count(b)) {
+            ops.push_back(Op{0, gi, b});
+            filled.insert(b);
+            dirty.erase(b);
+          }
+        }
+        ops.push_back(Op{1, gi, -1});
+        for (const Ver& v : g.outs) dirty.insert(buffer_id(E, v, par));
+      }
+      if (pass == 1) sched[par] = ops;
+    }
+  E->sched = sched;
+  E->fill_all.assign(all_fill.begin(), all_fill.end());
+}
+
+static void invalidate_graph(kf_exec* E) {
+  if (E->gexec) {
+    cudaGraphExecDestroy(E->gexec);
+    E->gexec = nullptr;
+  }
+}
+
+static void prepare_pointers(kf_exec* E, void* const* arrays, void* scratch, const double* params) {
+  const Program& p = E->prog->p;
+  std::vector<void*> arr(arrays, arrays + p.na);
+  std::vector<double> prm(params ? params : nullptr, params ? params + p.n_params : nullptr);
+  if (!params) prm.assign(p.n_params, 0.0);
+  if (!E->blobs_valid || arr != E->cur_arrays || scratch != E->cur_scratch || prm != E->cur_params) {
+    E->cur_arrays = arr;
+    E->cur_scratch = scratch;
+    E->cur_params = prm;
+    build_blobs(E);
+    invalidate_graph(E);
+  }
+}
+
+static void exec_run(kf_exec* E, void* const* arrays, void* scratch, uint64_t scratch_bytes, int64_t nsteps,
+                     const double* params, cudaStream_t s) {
+  const Program& p = E->prog->p;
+  if (!arrays) fail(KF_E_ARG, "arrays is NULL");
+  for (int x = 0; x < p.na; x++) {
+    if (!arrays[x]) fail(KF_E_ARG, "array pointer " + std::to_string(x) + " is NULL");
+    if (reinterpret_cast<uintptr_t>(arrays[x]) & 127) fail(KF_E_ARG, "array base pointers must be 128-byte aligned");
+  }
+  if (scratch_bytes < E->scratch_bytes || (E->scratch_bytes && !scratch))
+    fail(KF_E_RESOURCE, "scratch too small: need " + std::to_string(E->scratch_bytes) + " bytes");
+  if (nsteps < 0) fail(KF_E_ARG, "nsteps < 0");
+  if (p.n_params > 0 && !params) fail(KF_E_ARG, "params is NULL but the program has PARAM slots");
+  ensure_device(E);
+  prepare_pointers(E, arrays, scratch, params);
+  if (nsteps == 0) return;
+  // renamed copies share the array's ghost values (frozen boundaries, R9)
+  std::vector<void*> arr(arrays, arrays + p.na);
+  if (!E->scratch_vers.empty() && (E->shell_init_scratch != scratch || E->shell_init_arrays != arr)) {
+    Geom gm = geom(p);
+    for (size_t i = 0; i < E->scratch_vers.size(); i++)
+      CK(launch_copy_shell(buf_ptr(E, p.na + int(i)), arrays[E->scratch_vers[i].x], p.es, gm, s));
+    E->shell_init_scratch = scratch;
+    E->shell_init_arrays = arr;
+  }
+  for (int b : E->fill_all) run_fill(E, b, s);
+  int64_t reps = nsteps / E->period, rem = nsteps % E->period;
+  if (E->use_graph && !E->profiling && reps > 0) {
+    if (!E->gexec) {
+      if (!E->cap_stream) CK(cudaStreamCreateWithFlags(&E->cap_stream, cudaStreamNonBlocking));
+      cudaGraph_t graph;
+      CK(cudaStreamBeginCapture(E->cap_stream, cudaStreamCaptureModeThreadLocal));
+      try {
+        for (int par = 0; par < E->period; par++) run_step(E, par, E->cap_stream);
+      } catch (...) {
+        cudaStreamEndCapture(E->cap_stream, &graph);
+        throw;
+      }
+      CK(cudaStreamEndCapture(E->cap_stream, &graph));
+      CK(cudaGraphInstantiate(&E->gexec, graph, 0));
+      cudaGraphDestroy(graph);
+    }
+    for (int64_t r = 0; r < reps; r++) CK(cudaGraphLaunch(E->gexec, s));
+  } else {
+    for (int64_t r = 0; r < reps; r++)
+      for (int par = 0; par < E->period; par++) run_step(E, par, s);
+  }
+  for (int64_t r = 0; r < rem; r++) run_step(E, int(r), s);
+  // after an odd number of steps the renamed final versions sit in scratch: copy back
+  if (E->period == 2 && (nsteps % 2) == 1) {
+    for (int x = 0; x < p.na; x++)
+      if (p.relaxed[x] && p.step_live[x]) {
+        int b = buffer_id(E, Ver{x, int(p.writers[x].size())}, 0);
+        CK(cudaMemcpyAsync(arrays[x], buf_ptr(E, b), E->array_bytes, cudaMemcpyDeviceToDevice, s));
+      }
+  }
+  CK(cudaGetLastError());
+}
+
+}  // namespace kf
+
+extern "C" {
+
+kf_status kf_exec_create(kf_program* prog, const int32_t* plan, const kf_target* target, kf_exec** out) {
+  KF_TRY({
+    if (!prog || !plan || !out) fail(KF_E_ARG, "null argument");
+    check_target(target);
+    const Program& p = prog->p;
+    for (int k = 0; k < p.nk; k++)
+      if (plan[k] < 0) fail(KF_E_ILLEGAL_PLAN, "V1 PARTITION: kernel " + std::to_string(k) + " has no group");
+    auto E = std::make_unique<kf_exec>();
+    E->prog = prog;
+    E->t = *target;
+    E->plan = make_plan(p, plan);
+    kf_violation why{};
+    std::vector<GroupLowering> Ls;
+    int code = validate_plan(p, E->plan, *target, &why, &Ls);
+    if (code != KF_V_OK)
+      fail(KF_E_ILLEGAL_PLAN, "plan violates constraint V" + std::to_string(code) + " in group " + std::to_string(why.group));
+    E->order = quotient_order(p, E->plan);
+    // renamed versions -> scratch buffers ("redundant arrays")
+    for (int x = 0; x < p.na; x++) {
+      if (!p.relaxed[x]) continue;
+      int w = int(p.writers[x].size());
+      for (int v = 1; v <= w; v++) {
+        if (v == w && !p.step_live[x]) continue;   // final version of a TEMP array lives in the array itself
+        E->scratch_vers.push_back(Ver{x, v});
+      }
+      if (p.step_live[x]) E->period = 2;
+    }
+    E->array_bytes = uint64_t(p.layout.elems) * p.es;
+    E->array_bytes = (E->array_bytes + 255) / 256 * 256;
+    E->scratch_bytes = E->array_bytes * E->scratch_vers.size();
+    const int TZ = target->tile[2] > 0 ? std::min<int64_t>(target->tile[2], p.n[2]) : int(p.n[2]);
+    int64_t units = ((p.n[0] + target->tile[0] - 1) / target->tile[0]) * ((p.n[1] + target->tile[1] - 1) / target->tile[1]) *
+                    ((p.n[2] + TZ - 1) / TZ);
+    if (units > 2147483647) fail(KF_E_UNSUPPORTED, "grid too large");
+    E->G.resize(E->plan.m);
+    for (int gi = 0; gi < E->plan.m; gi++) {
+      GroupExec& g = E->G[gi];
+      g.gid = gi;
+      g.L = std::move(Ls[gi]);
+      g.cg = generate_group_kernel(p, g.L, gi);
+      g.grid = int(units);
+      g.smem = g.L.smem;
+      uint64_t rd, wr;
+      g.bytes = group_bytes(p, E->plan.groups[gi], &rd, &wr);
+      for (auto& r : g.L.rings) (r.live_in ? g.ins : g.mids).push_back(r.ver);
+      g.outs = g.L.live_out;
+      E->step_bytes += g.bytes;
+    }
+    // JIT all groups (NVRTC, sm_100a); identical sources are compiled once per process
+    for (auto& g : E->G) g.comp = compile_cached(g.cg.source, g.cg.name);
+    build_schedule(E.get());
+    *out = E.release();
+  });
+}
+
+void kf_exec_destroy(kf_exec* ex) {
+  if (!ex) return;
+  try {
+    invalidate_graph(ex);
+    if (ex->cap_stream) cudaStreamDestroy(ex->cap_stream);
+    for (auto& t : ex->pending) {
+      cudaEventDestroy(std::get<1>(t));
+      cudaEventDestroy(std::get<2>(t));
+    }
+    for (auto e : ex->evpool) cudaEventDestroy(e);
+    for (void* d : ex->dev_arrays) cudaFree(d);
+    if (ex->dev_scratch) cudaFree(ex->dev_scratch);
+  } catch (...) {
+  }
+  delete ex;
+}
+
+kf_status kf_exec_scratch_bytes(const kf_exec* ex, uint64_t* bytes) {
+  KF_TRY({
+    if (!ex || !bytes) fail(KF_E_ARG, "null argument");
+    *bytes = ex->scratch_bytes;
+  });
+}
+
+kf_status kf_exec_run(kf_exec* ex, void* const* arrays, void* scratch, uint64_t scratch_bytes, int64_t nsteps,
+                      const double* params, void* cuda_stream) {
+  KF_TRY({
+    if (!ex) fail(KF_E_ARG, "null exec");
+    exec_run(ex, arrays, scratch, scratch_bytes, nsteps, params, (cudaStream_t)cuda_stream);
+  });
+}
+
+kf_status kf_run_host(kf_exec* ex, void* const* host_arrays, int64_t nsteps, const double* params, void* cuda_stream,
+                      uint64_t* h2d_bytes, uint64_t* d2h_bytes) {
+  KF_TRY({
+    if (!ex || !host_arrays) fail(KF_E_ARG, "null argument");
+    const Program& p = ex->prog->p;
+    cudaStream_t s = (cudaStream_t)cuda_stream;
+    CK(cudaFree(nullptr));
+    if (ex->dev_arrays.empty()) {
+      for (int x = 0; x < p.na; x++) {
+        void* d = nullptr;
+        if (cudaMalloc(&d, ex->array_bytes) != cudaSuccess) fail(KF_E_OOM, "cudaMalloc failed in kf_run_host");
+        ex->dev_arrays.push_back(d);
+      }
+      if (ex->scratch_bytes && cudaMalloc(&ex->dev_scratch, ex->scratch_bytes) != cudaSuccess)
+        fail(KF_E_OOM, "cudaMalloc (scratch) failed in kf_run_host");
+      ex->host_first = true;
+    }
+    uint64_t h2d = 0, d2h = 0;
+    for (int x = 0; x < p.na; x++) {
+      // inputs of a step: arrays read before being written (upward-exposed) and read-only arrays;
+      // the first call also uploads every array (ghost values of temporaries)
+      bool input = !p.readers_of_version(x, 0).empty();
+      if (input || ex->host_first) {
+        CK(cudaMemcpyAsync(ex->dev_arrays[x], host_arrays[x], uint64_t(p.layout.elems) * p.es, cudaMemcpyHostToDevice, s));
+        h2d += uint64_t(p.layout.elems) * p.es;
+      }
+    }
+    ex->host_first = false;
+    exec_run(ex, ex->dev_arrays.data(), ex->dev_scratch, ex->scratch_bytes, nsteps, params, s);
+    for (int x = 0; x < p.na; x++)
+      if (p.step_live[x]) {
+        CK(cudaMemcpyAsync(host_arrays[x], ex->dev_arrays[x], uint64_t(p.layout.elems) * p.es, cudaMemcpyDeviceToHost, s));
+        d2h += uint64_t(p.layout.elems) * p.es;
+      }
+    CK(cudaStreamSynchronize(s));
+    if (h2d_bytes) *h2d_bytes = h2d;
+    if (d2h_bytes) *d2h_bytes = d2h;
+  });
+}
+
+kf_status kf_exec_get_info(const kf_exec* ex, kf_exec_info* out) {
+  KF_TRY({
+    if (!ex || !out) fail(KF_E_ARG, "null argument");
+    kf_exec_info r{};
+    r.n_groups = int(ex->G.size());
+    int fills = 0, launches = 0;
+    const Program& p = ex->prog->p;
+    int naxes = 0;
+    for (int a = 0; a < 3; a++) naxes += p.bc[a] == KF_BC_PERIODIC;
+    for (auto& sc : ex->sched)
+      for (auto& op : sc) {
+        if (op.kind == 0) fills += 1;
+        else launches += 1;
+      }
+    r.fills_per_step = fills * naxes / ex->period;
+    r.launches_per_step = launches / ex->period + r.fills_per_step;
+    r.period = ex->period;
+    r.compulsory_bytes_per_step = ex->step_bytes;
+    *out = r;
+  });
+}
+
+kf_status kf_exec_group_info(const kf_exec* ex, int32_t group, kf_group_info* out) {
+  KF_TRY({
+    if (!ex || !out) fail(KF_E_ARG, "null argument");
+    if (group < 0 || group >= int(ex->G.size())) fail(KF_E_ARG, "group out of range");
+    const GroupExec& g = ex->G[group];
+    kf_group_info r{};
+    r.group = group;
+    r.grid = g.grid;
+    r.threads = g.L.threads;
+    r.smem_bytes = g.smem;
+    r.regs = g.regs >= 0 ? g.regs : g.comp->regs_ptxas;
+    r.local_bytes = g.local >= 0 ? g.local : g.comp->spill;
+    r.n_kernels = int(g.L.kernels.size());
+    r.bytes_per_launch = g.bytes;
+    std::strncpy(r.name, g.cg.name.c_str(), sizeof(r.name) - 1);
+    *out = r;
+  });
+}
+
+kf_status kf_exec_group_source(const kf_exec* ex, int32_t group, char* buf, int64_t cap, int64_t* len) {
+  KF_TRY({
+    if (!ex || !len) fail(KF_E_ARG, "null argument");
+    if (group < 0 || group >= int(ex->G.size())) fail(KF_E_ARG, "group out of range");
+    const std::string& s = ex->G[group].cg.source;
+    *len = int64_t(s.size());
+    if (buf && cap > 0) {
+      int64_t n = std::min<int64_t>(cap - 1, int64_t(s.size()));
+      std::memcpy(buf, s.data(), size_t(n));
+      buf[n] = 0;
+    }
+  });
+}
+
+kf_status kf_exec_set_profiling(kf_exec* ex, int32_t on) {
+  KF_TRY({
+    if (!ex) fail(KF_E_ARG, "null exec");
+    for (auto& t : ex->pending) {   // drop unread measurements (e.g. of a warm-up)
+      cudaEventSynchronize(std::get<2>(t));
+      ex->evpool.push_back(std::get<1>(t));
+      ex->evpool.push_back(std::get<2>(t));
+    }
+    ex->pending.clear();
+    ex->profiling = on != 0;
+    ex->gms.assign(ex->G.size(), 0.0);
+    ex->launches = 0;
+  });
+}
+
+kf_status kf_exec_group_times(kf_exec* ex, double* ms, int32_t cap, int32_t* n, int64_t* launches) {
+  KF_TRY({
+    if (!ex || !n) fail(KF_E_ARG, "null argument");
+    if (ex->gms.size() != ex->G.size()) ex->gms.assign(ex->G.size(), 0.0);
+    for (auto& t : ex->pending) {
+      float f = 0.f;
+      CK(cudaEventSynchronize(std::get<2>(t)));
+      CK(cudaEventElapsedTime(&f, std::get<1>(t), std::get<2>(t)));
+      ex->gms[std::get<0>(t)] += f;
+      ex->evpool.push_back(std::get<1>(t));
+      ex->evpool.push_back(std::get<2>(t));
+    }
+    ex->pending.clear();
+    for (int i = 0; i < int(ex->gms.size()) && i < cap && ms; i++) ms[i] = ex->gms[i];
+    *n = int(ex->gms.size());
+    if (launches) *launches = ex->launches;
+  });
+}
+
+kf_status kf_exec_set_graph(kf_exec* ex, int32_t on) {
+  KF_TRY({
+    if (!ex) fail(KF_E_ARG, "null exec");
+    ex->use_graph = on != 0;
+  });
+}
+
+kf_status kf_flush_l2(void* buf, uint64_t bytes, void* cuda_stream) {
+  KF_TRY({
+    static unsigned v = 1;
+    CK(launch_flush(buf, (long long)bytes, v++, (cudaStream_t)cuda_stream));
+  });
+}
+
+kf_status kf_jit_check(const kf_program* prog, const int32_t* plan, const kf_target* target, int32_t group,
+                       int32_t* regs, int32_t* spill_bytes, char* log, int64_t cap) {
+  KF_TRY({
+    if (!prog || !plan || !target) fail(KF_E_ARG, "null argument");
+    check_target(target);
+    const Program& p = prog->p;
+    Plan pl = make_plan(p, plan);
+    if (group < 0 || group >= pl.m) fail(KF_E_ARG, "group out of range");
+    GroupLowering L = lower_group(p, pl.groups[group], *target);
+    if (getenv("KF_DEBUG")) fprintf(stderr, "jit_check: lowered\n");
+    Codegen cg = generate_group_kernel(p, L, group);
+    if (getenv("KF_DEBUG")) fprintf(stderr, "jit_check: generated %zu bytes\n", cg.source.size());
+    auto c = compile_cached(cg.source, cg.name);
+    if (regs) *regs = c->regs_ptxas;
+    if (spill_bytes) *spill_bytes = c->spill;
+    if (log && cap > 0) {
+      int64_t n = std::min<int64_t>(cap - 1, int64_t(c->log.size()));
+      std::memcpy(log, c->log.data(), size_t(n));
+      log[n] = 0;
+    }
+  });
+}
+
+}  // extern "C"

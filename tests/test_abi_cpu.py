@@ -1,0 +1,150 @@
+"""C-ABI library vs the oracle on CPU (no GPU): the library loads, exports every symbol
+include/kf.h declares, and its DAG, classes, legality verdicts (with the first violation),
+byte counts, extended regions and resource model match the oracle bit for bit."""
+import re
+
+import numpy as np
+import pytest
+
+from oracle import enum as En
+from oracle import graph as G
+from oracle import legality as L
+from workloads import programs as P
+from workloads.program import BC_FROZEN, BC_PERIODIC, DT_F32, PROG_RELAX_ALL, PROG_RELAX_EXPANDABLE
+
+kf = pytest.importorskip("paper_conf_sc_wahibm14_b200")
+
+
+def header_symbols():
+    src = open("include/kf.h").read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(kf_[a-z0-9_]+)\s*\(", src)))
+
+
+def test_library_exports_every_header_symbol():
+    import ctypes
+    lib = ctypes.CDLL(kf._abi.LIB_PATH)
+    syms = header_symbols()
+    assert len(syms) >= 25
+    for s in syms:
+        assert hasattr(lib, s), s
+    assert set(syms) <= set(kf._abi.SIGNATURES), set(syms) - set(kf._abi.SIGNATURES)
+
+
+def test_program_errors_are_reported():
+    from workloads.program import Builder
+    b = Builder("bad", DT_F32, (4, 4, 4), (1, 1, 1), (BC_FROZEN,) * 3)
+    u = b.array("u")
+    b.kernel("k", (u, u[1, 0, 0] + 1.0))          # reads u at an offset while writing it (R1)
+    with pytest.raises(kf.KfError, match="KF_E_PROGRAM"):
+        kf.Program(b.build())
+    b = Builder("bad2", DT_F32, (4, 4, 4), (1, 1, 1), (BC_FROZEN,) * 3)
+    u, v = b.array("u"), b.array("v")
+    b.kernel("k", (v, u[2, 0, 0]))                 # offset beyond ghost
+    with pytest.raises(kf.KfError, match="ghost"):
+        kf.Program(b.build())
+
+
+def check_program(desc, plans=None, target=None):
+    p = kf.Program(desc)
+    tgt_o = L.Target() if target is None else target[0]
+    tgt_k = kf.Target() if target is None else target[1]
+    assert p.edges() == G.edges(desc)
+    nk = len(desc.kernels)
+    reach = p.reach()
+    ref = G.closure(nk, G.edges(desc))
+    assert reach.tolist() == ref
+    for x in range(len(desc.arrays)):
+        ai = p.array_info(x)
+        assert ai.cls == G.array_class(desc, x)
+        assert bool(ai.relaxed) == G.relaxed(desc, x)
+        assert bool(ai.step_live) == G.step_live(desc, x)
+    for plan in (plans if plans is not None else En.restricted_growth(nk)):
+        v_k = p.validate(plan, tgt_k)
+        v_o = L.validate(desc, plan, tgt_o)
+        assert v_k == v_o, (plan, v_k, v_o)
+        per_k, tb_k, tt_k = p.project(plan, tgt_k)
+        per_o, tb_o, tt_o = L.project(desc, plan, tgt_o)
+        assert tb_k == tb_o and tt_k == tt_o
+        for gk, go in zip(per_k, per_o):
+            assert (gk.bytes_read, gk.bytes_written) == (go[0], go[1])
+        for gi, grp in enumerate(L.groups_of(plan)):
+            s_o = L.schedule(desc, grp, tgt_o)
+            s_k = p.schedule(plan, gi, tgt_k)
+            assert per_k[gi].smem_bytes == s_o["smem"] and per_k[gi].regs_est == s_o["regs"]
+            for sk in s_k:
+                e = s_o["ext"][sk.kernel]
+                assert bool(sk.alive) == (e is not None)
+                if e is not None:
+                    assert (tuple(sk.elo), tuple(sk.ehi)) == e
+                    assert sk.delay == s_o["delay"][sk.kernel]
+    return p
+
+
+def test_tiny_fig3_pins_through_abi():
+    check_program(P.tiny())
+    p = check_program(P.fig3())
+    assert p.count_legal() == len(En.legal_plans(P.fig3())) == 20
+    plan, b = p.search(kf.SEARCH_BRUTE)
+    bo, bb = En.best_plan(P.fig3())
+    assert plan == bo == P.FIG3_PLAN_XY and b == bb        # the paper's X, Y fusion is the optimum
+    for nk in (4, 5, 6):
+        assert kf.Program(P.pointwise_chain(nk)).count_legal() == 2 ** (nk - 1)
+        assert kf.Program(P.shared_readonly(nk)).count_legal() == En.bell(nk)
+        assert kf.Program(P.disjoint(nk)).count_legal() == 1
+
+
+@pytest.mark.parametrize("seed", range(24))
+def test_random_programs_match_oracle(seed):
+    rng = np.random.default_rng(seed)
+    bc = tuple(int(x) for x in rng.integers(0, 2, size=3))
+    flags = [0, PROG_RELAX_EXPANDABLE, PROG_RELAX_ALL][seed % 3]
+    desc = P.random_program(seed, nk=5, na=4, bc=bc, flags=flags, max_r=1 + seed % 2)
+    check_program(desc)
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_search_equals_brute_force(seed):
+    desc = P.random_program(50 + seed, nk=6, na=4)
+    p = kf.Program(desc)
+    plan, b = p.search(kf.SEARCH_BRUTE)
+    bo, bb = En.best_plan(desc)
+    assert b == bb and plan == bo
+    assert p.count_legal() == len(En.legal_plans(desc))
+    g, gb = p.search(kf.SEARCH_GREEDY)
+    assert p.validate(g)[0] == 0 and gb >= b
+
+
+def test_resource_limits_V7_V8():
+    desc = P.tiny()
+    tk = kf.Target(smem_per_block=19983)
+    to = L.Target(smem_per_block=19983)
+    check_program(desc, target=(to, tk))
+    assert kf.Program(desc).validate([0, 0, 1], tk)[0] == L.V7_SMEM
+    tk = kf.Target(regs_per_thread_max=40)
+    to = L.Target(regs_per_thread_max=40)
+    check_program(desc, target=(to, tk))
+
+
+def test_weather_program_abi_and_greedy():
+    desc = P.weather(n=(16, 16, 8))
+    p = kf.Program(desc)
+    assert p.edges() == G.edges(desc)
+    unf = p.project(list(range(44)))[1]
+    assert unf == L.unfused_bytes(desc) == 142 * desc.npts * 8
+    plan, b = p.search(kf.SEARCH_GREEDY)
+    assert p.validate(plan) == L.validate(desc, plan)
+    assert p.validate(plan)[0] == 0 and b < unf
+    assert L.project(desc, plan)[1] == b
+
+
+def test_codegen_compiles_for_sm100a():
+    """NVRTC JIT of generated group kernels (no GPU needed): no spills, regs within the model."""
+    for desc, plan in ((P.tiny(), [0, 0, 1]), (P.fig3(), P.FIG3_PLAN_XY)):
+        p = kf.Program(desc)
+        per, _, _ = p.project(plan)
+        for g in range(len(per)):
+            regs, spill, log = p.jit_check(plan, g)
+            assert "sm_100a" in log
+            assert spill == 0
+            assert 0 < regs <= per[g].regs_est, (regs, per[g].regs_est)

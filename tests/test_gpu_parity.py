@@ -1,0 +1,132 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the oracle, element by element.
+
+fp64 bit-exact, fp32 within 2e-6 normwise and in practice bit-exact (north_star).
+Sizes span several tiles with ragged tails; full BASELINE sizes are checked on sampled
+windows (tests/test_gpu_fullsize.py)."""
+import numpy as np
+import pytest
+
+from oracle import enum as En
+from oracle import interp
+from oracle import legality as L
+from workloads import data as D
+from workloads import programs as P
+from workloads.program import BC_FROZEN, BC_PERIODIC, DT_F32, DT_F64, PROG_RELAX_ALL, PROG_RELAX_EXPANDABLE
+
+from .gpu_util import compare, run_kf
+
+pytestmark = pytest.mark.gpu
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():
+    pytest.skip("needs a GPU", allow_module_level=True)
+
+import paper_conf_sc_wahibm14_b200 as kf  # noqa: E402
+
+
+def test_tiny_config1_all_legal_plans():
+    """BASELINE config 1: 32^3 fp32, 4 steps, every legal plan (unfused and {K1,K2}{K3})."""
+    desc = P.tiny()
+    inputs = D.uniform(desc, 1)
+    ref = interp.run(desc, inputs, 4)
+    plans = En.legal_plans(desc)
+    assert len(plans) == 2
+    for plan in plans:
+        got, _ = run_kf(desc, plan, inputs, 4)
+        assert compare(desc, got, ref) == [], plan
+
+
+def test_tiny_closed_form_on_gpu():
+    desc = P.tiny()
+    inputs = D.quadratic(desc)
+    got, _ = run_kf(desc, [0, 0, 1], inputs, 1)
+    g = desc.ghost
+    w = got["w"][g[2] + 1:-g[2] - 1, g[1] + 1:-g[1] - 1, g[0] + 1:-g[0] - 1]
+    assert np.all(w == 0.0)                       # L7(L7(quadratic)) = L7(12) = 0 away from the boundary
+    assert compare(desc, got, interp.run(desc, inputs, 1)) == []
+
+
+@pytest.mark.parametrize("tile", [(32, 16, 0), (16, 8, 0), (32, 16, 7), (8, 8, 5)])
+def test_tiny_ragged_tiles_and_z_chunks(tile):
+    desc = P.tiny(n=(37, 21, 19))
+    inputs = D.uniform(desc, 2)
+    ref = interp.run(desc, inputs, 3)
+    got, _ = run_kf(desc, [0, 0, 1], inputs, 3, kf.Target(tile=tile))
+    assert compare(desc, got, ref) == []
+
+
+def test_fig3_all_20_legal_plans_fp64():
+    """Fig. 3 kernels in fp64: every legal plan, including the paper's X,Y, bit-exact."""
+    desc = P.fig3(n=(40, 24, 10))
+    inputs = D.inputs_for(desc, 3)
+    ref = interp.run(desc, inputs, 1)
+    plans = En.legal_plans(desc)
+    assert len(plans) == 20
+    for plan in plans:
+        got, _ = run_kf(desc, plan, inputs, 1)
+        assert compare(desc, got, ref) == [], plan
+
+
+@pytest.mark.parametrize("seed", range(16))
+def test_random_programs_random_legal_plans(seed):
+    rng = np.random.default_rng(1000 + seed)
+    bc = tuple(int(x) for x in rng.integers(0, 2, size=3))
+    flags = [0, PROG_RELAX_EXPANDABLE, PROG_RELAX_ALL][seed % 3]
+    dtype = DT_F32 if seed % 2 else DT_F64
+    n = tuple(int(x) for x in rng.integers(9, 40, size=3))
+    desc = P.random_program(2000 + seed, nk=5, na=4, n=n, dtype=dtype, bc=bc, flags=flags, max_r=1 + seed % 2)
+    inputs = D.uniform(desc, seed)
+    nsteps = 1 + seed % 3
+    ref = interp.run(desc, inputs, nsteps)
+    legal = En.legal_plans(desc)
+    pick = [legal[i] for i in sorted(set(rng.integers(0, len(legal), size=4).tolist()))]
+    tile = [(32, 16, 0), (16, 16, 0), (8, 4, 6), (32, 8, 11)][seed % 4]
+    for plan in pick:
+        got, _ = run_kf(desc, plan, inputs, nsteps, kf.Target(tile=tile))
+        assert compare(desc, got, ref) == [], (plan, tile)
+
+
+def test_weather_small_fp64_plans():
+    """Config 3 program at a small size: unfused, the hand plan and the searched plan, 2 steps."""
+    from .test_oracle import weather_hand_plan
+    desc = P.weather(n=(48, 40, 12))
+    inputs = D.inputs_for(desc, 3)
+    ref = interp.run(desc, inputs, 2)
+    plan_g, _ = kf.Program(desc).search(kf.SEARCH_GREEDY)
+    for plan in (list(range(44)), weather_hand_plan(desc), plan_g):
+        got, _ = run_kf(desc, plan, inputs, 2)
+        assert compare(desc, got, ref) == [], plan
+
+
+def test_graph_and_eager_agree_and_odd_even_steps():
+    desc = P.weather(n=(32, 32, 8))
+    inputs = D.inputs_for(desc, 5)
+    plan, _ = kf.Program(desc).search(kf.SEARCH_GREEDY)
+    for nsteps in (1, 2, 3):
+        ref = interp.run(desc, inputs, nsteps)
+        for graph in (True, False):
+            got, _ = run_kf(desc, plan, inputs, nsteps, graph=graph)
+            assert compare(desc, got, ref) == [], (nsteps, graph)
+
+
+def test_registers_within_model_and_no_spills():
+    """V8's register model must bound ptxas (R20); no local-memory spills."""
+    desc = P.weather(n=(64, 64, 16))
+    plan, _ = kf.Program(desc).search(kf.SEARCH_GREEDY)
+    _, ex = run_kf(desc, plan, D.inputs_for(desc, 1), 1)
+    per, _, _ = kf.Program(desc).project(plan)
+    for g in range(ex.info().n_groups):
+        gi = ex.group_info(g)
+        assert gi.local_bytes == 0, gi.name
+        assert gi.regs <= per[g].regs_est, (gi.name, gi.regs, per[g].regs_est)
+
+
+def test_run_host_path():
+    desc = P.tiny(n=(24, 20, 16))
+    inputs = D.uniform(desc, 9)
+    prog = kf.Program(desc)
+    ex = kf.Exec(prog, [0, 0, 1])
+    host = [torch.from_numpy(prog.to_device_layout(inputs[nm])).pin_memory() for nm, _ in desc.arrays]
+    h2d, d2h = ex.run_host([t.data_ptr() for t in host], 3)
+    got = {nm: prog.from_device_layout(t.numpy()) for (nm, _), t in zip(desc.arrays, host)}
+    assert compare(desc, got, interp.run(desc, inputs, 3)) == []
+    assert h2d > 0 and d2h > 0
