@@ -204,7 +204,11 @@ def schedule(prog: Program, grp: List[int], target: Target):
         span = A - B + 1
         slots = span + S - 1
         (lo, hi) = boxes[(x, v)]
-        res.append(("in", x, v, TX + lo[0] + hi[0], TY + lo[1] + hi[1], slots, A, B))
+        # the TMA box of a live-in starts on a 16-byte boundary in x (R20a): lower x extent rounded
+        # up to a multiple of 16/es elements (toward +inf, also when negative)
+        al = 16 // es
+        lox = -((-lo[0]) // al) * al
+        res.append(("in", x, v, TX + lox + hi[0], TY + lo[1] + hi[1], slots, A, B))
     for p in alive:
         for x in G.writes(prog, p):
             v = G.version_written(prog, p, x)

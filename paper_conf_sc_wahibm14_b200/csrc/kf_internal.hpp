@@ -105,6 +105,8 @@ struct Ring {
   bool live_in = false;   // staged by TMA from HBM; else produced in the group
   int producer = -1;      // kernel producing it (in-group rings)
   int blo[3], bhi[3];     // box extents beyond T (xy used for SMEM; z for plane range)
+  int ax_lo = 0;          // x extent below T of the SMEM box: live-in boxes start on a 16-byte
+                          // boundary (TMA faults on unaligned x starts, measured on B200)
   int wx, hy, px;         // box width, height, padded row pitch (elements)
   int plane_bytes;        // roundup(px*hy*es, 128)
   int slots;              // ring depth

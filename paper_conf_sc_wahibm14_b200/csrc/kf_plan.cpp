@@ -131,7 +131,11 @@ GroupLowering lower_group(const Program& p, const std::vector<int>& g, const kf_
   }
   const int es = p.es, TX = t.tile[0], TY = t.tile[1], S = t.stages;
   auto finish_ring = [&](Ring& r) {
-    r.wx = TX + r.blo[0] + r.bhi[0];
+    const int a = 16 / es;
+    // TMA box x start must be 16-byte aligned: round the lower x extent of a live-in box up to a
+    // multiple of 16/es elements (ceil toward +inf also for negative extents).
+    r.ax_lo = r.live_in ? (r.blo[0] >= 0 ? (r.blo[0] + a - 1) / a * a : -((-r.blo[0]) / a * a)) : r.blo[0];
+    r.wx = TX + r.ax_lo + r.bhi[0];
     r.hy = TY + r.blo[1] + r.bhi[1];
     r.px = int(rup(r.wx, 16 / es));
     r.plane_bytes = int(rup(int64_t(r.px) * r.hy * es, 128));
@@ -379,6 +383,7 @@ void check_target(const kf_target* t) {
   if (t->tile[0] < 1 || t->tile[1] < 1 || t->tile[2] < 0 || t->tile[0] > 224 || t->tile[1] > 224)
     fail(KF_E_ARG, "tile must be TX,TY in [1,224], TZ >= 0");
   if (t->max_halo < 0 || t->max_halo > 16) fail(KF_E_ARG, "max_halo must be in [0,16] (TMA box <= 256)");
+  if (t->tile[0] % 4) fail(KF_E_ARG, "tile TX must be a multiple of 4 (16-byte aligned TMA boxes)");
   if (t->stages < 2 || t->stages > 8) fail(KF_E_ARG, "stages must be in [2, 8]");
   if (t->threads < 32 || t->threads > 1024 || t->threads % 32) fail(KF_E_ARG, "threads must be a multiple of 32 in [32,1024]");
   if (!(t->hbm_bytes_per_s > 0)) fail(KF_E_ARG, "hbm_bytes_per_s must be > 0");

@@ -102,6 +102,11 @@ static Compiled nvrtc_compile(const std::string& src, const std::string& name) {
   c.cubin.resize(cs);
   nvrtcGetCUBIN(prog, c.cubin.data());
   nvrtcDestroyProgram(&prog);
+  if (const char* dir = getenv("KF_DUMP_DIR")) {   // debugging aid: keep the generated source and cubin
+    std::string base = std::string(dir) + "/" + name;
+    if (FILE* f = fopen((base + ".cu").c_str(), "w")) { fwrite(src.data(), 1, src.size(), f); fclose(f); }
+    if (FILE* f = fopen((base + ".cubin").c_str(), "wb")) { fwrite(c.cubin.data(), 1, c.cubin.size(), f); fclose(f); }
+  }
   auto p = c.log.find("Used ");
   if (p != std::string::npos) c.regs_ptxas = atoi(c.log.c_str() + p + 5);
   auto q = c.log.find("bytes spill stores");
@@ -248,6 +253,10 @@ static void build_blobs(kf_exec* E) {
         cuuint32_t box[3] = {cuuint32_t(R.px), cuuint32_t(R.hy), 1};
         cuuint32_t estr[3] = {1, 1, 1};
         CUtensorMap* tm = reinterpret_cast<CUtensorMap*>(base + 128 * i);
+        if (getenv("KF_DEBUG"))
+          fprintf(stderr, "tmap g%d in%zu ptr=%p dims=%llu,%llu,%llu strides=%llu,%llu box=%u,%u,%u\n", g.gid, i, ptr,
+                  (unsigned long long)dims[0], (unsigned long long)dims[1], (unsigned long long)dims[2],
+                  (unsigned long long)strides[0], (unsigned long long)strides[1], box[0], box[1], box[2]);
         ckd(drv().tensorMapEncodeTiled(tm, es == 4 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3,
                                        ptr, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
                                        CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
@@ -280,6 +289,11 @@ static void launch_group(kf_exec* E, int gi, int par, cudaStream_t s) {
   if (blob.size() > sizeof(tmp)) fail(KF_E_RESOURCE, "kernel argument block too large");
   std::memcpy(tmp, blob.data(), blob.size());
   void* params[] = {tmp};
+  if (getenv("KF_DEBUG")) {
+    fprintf(stderr, "launch %s grid=%d threads=%d smem=%d blob=%zu:", g.cg.name.c_str(), g.grid, g.L.threads, g.smem, blob.size());
+    for (size_t i = 0; i < blob.size(); i += 8) fprintf(stderr, " %016llx", *(unsigned long long*)(tmp + i));
+    fprintf(stderr, "\n");
+  }
   ckd(drv().launchKernel(g.fn, g.grid, 1, 1, g.L.threads, 1, 1, g.smem, (CUstream)s, params, nullptr),
       ("cuLaunchKernel " + g.cg.name).c_str());
 }
