@@ -59,6 +59,9 @@ def choose_plan(prog, target, which: str):
     n = prog.nk
     if which == "unfused":
         return list(range(n)), "unfused (singletons)"
+    if which == "hand":
+        from workloads.programs import weather_hand_plan
+        return weather_hand_plan(prog.desc), "hand plan (App. A.4)"
     method = kf.SEARCH_BRUTE if n <= 10 else kf.SEARCH_GREEDY
     plan, _ = prog.search(method, target)
     return plan, ("brute-force optimum" if method == kf.SEARCH_BRUTE else "greedy search")
@@ -282,11 +285,12 @@ def run_kf(args):
     # dominant kernel = the group with the largest device time
     g_dom = int(np.argmax(gms))
     gi = ex.group_info(g_dom)
+    gname = gi.name.decode() if isinstance(gi.name, bytes) else gi.name
     launches_dom = args.steps * info.period // info.period
     t_launch_ms = gms[g_dom] / args.steps
     achieved = gi.bytes_per_launch / (t_launch_ms / 1e3) / 1e9
     roofline = {"bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s", "frac": achieved / hbm_peak,
-                "traffic": ncu_traffic(gi.name), "kernel": gi.name, "peak_source": peak_src,
+                "traffic": ncu_traffic(gname), "kernel": gname, "peak_source": peak_src,
                 "share_of_step": gms[g_dom] / max(1e-9, sum(gms)),
                 "algorithmic_bytes_per_launch": gi.bytes_per_launch,
                 "per_group_ms_per_step": [g / args.steps for g in gms]}
@@ -373,7 +377,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="kf", choices=["kf", "reference"])
     ap.add_argument("--workload", default="weather")
-    ap.add_argument("--plan", default="best", choices=["best", "unfused"])
+    ap.add_argument("--plan", default="best", choices=["best", "unfused", "hand"])
     ap.add_argument("--tile", default=None)
     ap.add_argument("--stages", type=int, default=None)
     ap.add_argument("--threads", type=int, default=None)

@@ -242,7 +242,10 @@ kf_status kf_exec_scratch_bytes(const kf_exec* ex, uint64_t* bytes);
  * default stream).  arrays: n_arrays device pointers to the *allocation base* of each
  * array (kf_array_layout).  params: n_params values (NULL if none).  After the call
  * completes, every array that is not TEMP (written but not step-live, R15) holds its
- * post-nsteps value; TEMP contents are unspecified.  Read-only arrays are never written.
+ * post-nsteps value in the interior; TEMP contents are unspecified.  Ghost cells of FROZEN
+ * axes are never written; ghost layers of PERIODIC axes are overwritten with wrapped copies
+ * of the interior (their contents after a run are the wrap of some step's values).
+ * Read-only arrays' interiors are never written.
  * Errors: KF_E_ARG, KF_E_RESOURCE (scratch too small), KF_E_CUDA (launch failure; async
  * faults surface at the next synchronising call). */
 kf_status kf_exec_run(kf_exec* ex, void* const* arrays, void* scratch, uint64_t scratch_bytes,

@@ -87,7 +87,7 @@ def test_random_programs_random_legal_plans(seed):
 
 def test_weather_small_fp64_plans():
     """Config 3 program at a small size: unfused, the hand plan and the searched plan, 2 steps."""
-    from .test_oracle import weather_hand_plan
+    from workloads.programs import weather_hand_plan
     desc = P.weather(n=(48, 40, 12))
     inputs = D.inputs_for(desc, 3)
     ref = interp.run(desc, inputs, 2)

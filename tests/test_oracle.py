@@ -385,27 +385,7 @@ def test_weather_greedy_plan_shape_legal():
     assert fused < 142
 
 
-def weather_hand_plan(prog):
-    kn = [k.name for k in prog.kernels]
-    g = {}
-    lab = 0
-
-    def grp(names):
-        nonlocal lab
-        for s in names:
-            g[s] = lab
-        lab += 1
-    grp(["velx", "vely", "velz", "pott", "pres"])
-    for phi in ("DENS", "MOMX", "MOMY", "MOMZ", "RHOT"):
-        grp([f"flxx_{phi}", f"flxy_{phi}", f"flxz_{phi}", f"div_{phi}"])
-    grp(["pgx", "pgy", "pgz", "corx", "cory"])
-    grp(["lap_VELX", "difx"])
-    grp(["lap_VELY", "dify"])
-    grp(["lap_VELZ", "difz"])
-    grp(["lap_POTT", "lap2", "dift"])
-    for phi in ("DENS", "MOMX", "MOMY", "MOMZ", "RHOT"):
-        grp([f"rk_{phi}"])
-    return [g[s] for s in kn]
+from workloads.programs import weather_hand_plan  # noqa: E402
 
 
 # ------------------------------------------------------------------ O-6 bytes / O-9 projection
