@@ -1,0 +1,51 @@
+"""Sweep tile/stages/threads for a plan of the weather workload in one process (inputs generated once)."""
+import itertools, json, os, sys, time
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch
+import paper_conf_sc_wahibm14_b200 as kf
+from workloads import programs as P, data as D
+
+def main():
+    plan_kind = sys.argv[1] if len(sys.argv) > 1 else "hand"
+    configs = json.loads(sys.argv[2]) if len(sys.argv) > 2 else [[[32, 16, 0], 2, 256]]
+    desc = P.weather(n=(512, 512, 128))
+    prog = kf.Program(desc)
+    inputs = D.weather_inputs(desc, 3)
+    dev = kf.device_arrays(prog, inputs)
+    del inputs
+    out = []
+    for tile, stages, threads in configs:
+        tgt = kf.Target(tile=tile, stages=stages, threads=threads)
+        if plan_kind == "hand":
+            plan = P.weather_hand_plan(desc)
+        elif plan_kind == "unfused":
+            plan = list(range(44))
+        else:
+            plan, _ = prog.search(kf.SEARCH_GREEDY, tgt)
+        try:
+            ex = kf.Exec(prog, plan, tgt)
+        except Exception as e:
+            print(json.dumps({"tile": tile, "stages": stages, "threads": threads, "error": str(e)[:200]}), flush=True)
+            continue
+        sb = ex.scratch_bytes()
+        scr = torch.empty(sb, dtype=torch.uint8, device="cuda") if sb else None
+        ex.run(dev, scr, 3)
+        torch.cuda.synchronize()
+        ex.set_profiling(True)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        ex.run(dev, scr, 10)
+        e1.record()
+        torch.cuda.synchronize()
+        ms = e0.elapsed_time(e1) / 10
+        gms, _ = ex.group_times()
+        info = ex.info()
+        r = {"tile": tile, "stages": stages, "threads": threads, "ms_per_step": ms,
+             "TBps": info.compulsory_bytes_per_step / ms / 1e9,
+             "groups": [(ex.group_info(g).name.decode(), round(gms[g] / 10, 4),
+                         round(ex.group_info(g).bytes_per_launch / (gms[g] / 10) / 1e9, 2),
+                         ex.group_info(g).smem_bytes, ex.group_info(g).regs) for g in range(len(gms))]}
+        print(json.dumps(r), flush=True)
+        del ex, scr
+
+main()
