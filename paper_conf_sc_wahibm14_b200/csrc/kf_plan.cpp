@@ -199,6 +199,17 @@ GroupLowering lower_group(const Program& p, const std::vector<int>& g, const kf_
   }
   L.mbar_off = off;
   L.smem = off + 8 * S + 128;
+  // threads per CTA: enough to cover the largest extended region in one pass (a region just
+  // above the thread count would otherwise take a second, nearly empty round), within [threads, 512]
+  {
+    int maxr = 0;
+    for (int k : alive) {
+      const Ext& e = L.ext[k];
+      maxr = std::max(maxr, (TX + e.elo[0] + e.ehi[0]) * (TY + e.elo[1] + e.ehi[1]));
+    }
+    int nt = (maxr + 31) / 32 * 32;
+    L.threads = (nt > t.threads && nt <= 512) ? nt : t.threads;
+  }
   int depth = 1;
   for (int k : g) depth = std::max(depth, p.kernels[k].depth);
   L.depth = depth;
