@@ -41,6 +41,7 @@ class Target:
     threads: int = 256
     max_halo: int = 16
     internal_axes: int = 0          # bitmask of axes split across ranks (treated like periodic by V6)
+    zunroll: int = 2                # planes per stream iteration U (ring depth grows with U, R20)
 
 
 # ---------------------------------------------------------------- plans
@@ -202,7 +203,7 @@ def schedule(prog: Program, grp: List[int], target: Target):
                 if x in G.writes(prog, b) and (x, G.version_written(prog, x=x, k=b)) in lout:
                     A = max(A, -D[b])
         span = A - B + 1
-        slots = span + S - 1
+        slots = span + target.zunroll * (S - 1)
         (lo, hi) = boxes[(x, v)]
         # the TMA box of a live-in starts on a 16-byte boundary in x (R20a): lower x extent rounded
         # up to a multiple of 16/es elements (toward +inf, also when negative)
@@ -216,7 +217,7 @@ def schedule(prog: Program, grp: List[int], target: Target):
                   and G.version_read(prog, c, x) == v]
             if not rd:
                 continue
-            span = max(D[c] - d[2] for c, offs in rd for d in offs) - D[p] + 1
+            span = max(D[c] - d[2] for c, offs in rd for d in offs) - D[p] + 1 + (target.zunroll - 1)
             (lo, hi) = ext[p]
             res.append(("mid", x, v, TX + lo[0] + hi[0], TY + lo[1] + hi[1], span, 0, 0))
     smem = 0

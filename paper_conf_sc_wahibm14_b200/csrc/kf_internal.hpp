@@ -124,7 +124,7 @@ struct GroupLowering {
   int smem = 0, regs = 0, depth = 0;
   int mbar_off = 0;
   int tile[3];
-  int stages = 2, threads = 256;
+  int stages = 2, threads = 256, zunroll = 1;
   int ring_of(const Ver& v) const;        // index in rings or -1
 };
 

@@ -74,6 +74,7 @@ GroupLowering lower_group(const Program& p, const std::vector<int>& g, const kf_
   L.tile[2] = t.tile[2];
   L.stages = t.stages;
   L.threads = t.threads;
+  L.zunroll = t.zunroll;
   L.live_in = group_live_in(p, g);
   L.live_out = group_live_out(p, g);
   L.live_out_set = std::set<Ver>(L.live_out.begin(), L.live_out.end());
@@ -129,7 +130,7 @@ GroupLowering lower_group(const Program& p, const std::vector<int>& g, const kf_
     }
     L.delay[k] = dk;
   }
-  const int es = p.es, TX = t.tile[0], TY = t.tile[1], S = t.stages;
+  const int es = p.es, TX = t.tile[0], TY = t.tile[1], S = t.stages, U = t.zunroll;
   auto finish_ring = [&](Ring& r) {
     const int a = 16 / es;
     // TMA box x start must be 16-byte aligned: round the lower x extent of a live-in box up to a
@@ -169,7 +170,7 @@ GroupLowering lower_group(const Program& p, const std::vector<int>& g, const kf_
           A = std::max(A, -L.delay[b]);
     r.A = A;
     r.B = B;
-    r.slots = (A - B + 1) + S - 1;
+    r.slots = (A - B + 1) + U * (S - 1);
     finish_ring(r);
     L.rings.push_back(r);
   }
@@ -187,7 +188,7 @@ GroupLowering lower_group(const Program& p, const std::vector<int>& g, const kf_
       r.live_in = false;
       r.producer = pk;
       for (int a = 0; a < 3; a++) { r.blo[a] = L.ext[pk].elo[a]; r.bhi[a] = L.ext[pk].ehi[a]; }
-      r.slots = mx - L.delay[pk] + 1;
+      r.slots = mx - L.delay[pk] + 1 + (U - 1);
       finish_ring(r);
       L.rings.push_back(r);
     }
@@ -396,6 +397,7 @@ void check_target(const kf_target* t) {
   if (t->max_halo < 0 || t->max_halo > 16) fail(KF_E_ARG, "max_halo must be in [0,16] (TMA box <= 256)");
   if (t->tile[0] % 4) fail(KF_E_ARG, "tile TX must be a multiple of 4 (16-byte aligned TMA boxes)");
   if (t->stages < 2 || t->stages > 8) fail(KF_E_ARG, "stages must be in [2, 8]");
+  if (t->zunroll < 1 || t->zunroll > 4) fail(KF_E_ARG, "zunroll must be in [1, 4]");
   if (t->threads < 32 || t->threads > 1024 || t->threads % 32) fail(KF_E_ARG, "threads must be a multiple of 32 in [32,1024]");
   if (!(t->hbm_bytes_per_s > 0)) fail(KF_E_ARG, "hbm_bytes_per_s must be > 0");
 }

@@ -340,6 +340,7 @@ kf_status kf_target_b200(kf_target* out) {
     t.threads = 256;
     t.max_halo = 16;
     t.internal_axes = 0;
+    t.zunroll = 2;
     *out = t;
   });
 }

@@ -46,11 +46,12 @@ def test_tiny_closed_form_on_gpu():
 
 
 @pytest.mark.parametrize("tile", [(32, 16, 0), (16, 8, 0), (32, 16, 7), (8, 8, 5)])
-def test_tiny_ragged_tiles_and_z_chunks(tile):
+@pytest.mark.parametrize("zunroll", [1, 2, 3])
+def test_tiny_ragged_tiles_and_z_chunks(tile, zunroll):
     desc = P.tiny(n=(37, 21, 19))
     inputs = D.uniform(desc, 2)
     ref = interp.run(desc, inputs, 3)
-    got, _ = run_kf(desc, [0, 0, 1], inputs, 3, kf.Target(tile=tile))
+    got, _ = run_kf(desc, [0, 0, 1], inputs, 3, kf.Target(tile=tile, zunroll=zunroll))
     assert compare(desc, got, ref) == []
 
 
@@ -80,8 +81,9 @@ def test_random_programs_random_legal_plans(seed):
     legal = En.legal_plans(desc)
     pick = [legal[i] for i in sorted(set(rng.integers(0, len(legal), size=4).tolist()))]
     tile = [(32, 16, 0), (16, 16, 0), (8, 4, 6), (32, 8, 11)][seed % 4]
+    zu = [1, 2, 3][seed % 3]
     for plan in pick:
-        got, _ = run_kf(desc, plan, inputs, nsteps, kf.Target(tile=tile))
+        got, _ = run_kf(desc, plan, inputs, nsteps, kf.Target(tile=tile, zunroll=zu))
         assert compare(desc, got, ref) == [], (plan, tile)
 
 
@@ -93,8 +95,9 @@ def test_weather_small_fp64_plans():
     ref = interp.run(desc, inputs, 2)
     plan_g, _ = kf.Program(desc).search(kf.SEARCH_GREEDY)
     for plan in (list(range(44)), weather_hand_plan(desc), plan_g):
-        got, _ = run_kf(desc, plan, inputs, 2)
-        assert compare(desc, got, ref) == [], plan
+        for zu in (1, 2):
+            got, _ = run_kf(desc, plan, inputs, 2, kf.Target(tile=(32, 8, 0), zunroll=zu))
+            assert compare(desc, got, ref) == [], (plan, zu)
 
 
 def test_graph_and_eager_agree_and_odd_even_steps():

@@ -14,8 +14,10 @@ def main():
     dev = kf.device_arrays(prog, inputs)
     del inputs
     out = []
-    for tile, stages, threads in configs:
-        tgt = kf.Target(tile=tile, stages=stages, threads=threads)
+    for cfg in configs:
+        tile, stages, threads = cfg[:3]
+        zu = cfg[3] if len(cfg) > 3 else 2
+        tgt = kf.Target(tile=tile, stages=stages, threads=threads, zunroll=zu)
         if plan_kind == "hand":
             plan = P.weather_hand_plan(desc)
         elif plan_kind == "unfused":
@@ -40,7 +42,7 @@ def main():
         ms = e0.elapsed_time(e1) / 10
         gms, _ = ex.group_times()
         info = ex.info()
-        r = {"tile": tile, "stages": stages, "threads": threads, "ms_per_step": ms,
+        r = {"tile": tile, "stages": stages, "threads": threads, "zunroll": zu, "ms_per_step": ms,
              "TBps": info.compulsory_bytes_per_step / ms / 1e9,
              "groups": [(ex.group_info(g).name.decode(), round(gms[g] / 10, 4),
                          round(ex.group_info(g).bytes_per_launch / (gms[g] / 10) / 1e9, 2),
