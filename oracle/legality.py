@@ -203,7 +203,7 @@ def schedule(prog: Program, grp: List[int], target: Target):
                 if x in G.writes(prog, b) and (x, G.version_written(prog, x=x, k=b)) in lout:
                     A = max(A, -D[b])
         span = A - B + 1
-        slots = span + target.zunroll * (S - 1)
+        slots = span + target.zunroll * S - 1      # U planes in use + U*(S-1) prefetched
         (lo, hi) = boxes[(x, v)]
         # the TMA box of a live-in starts on a 16-byte boundary in x (R20a): lower x extent rounded
         # up to a multiple of 16/es elements (toward +inf, also when negative)

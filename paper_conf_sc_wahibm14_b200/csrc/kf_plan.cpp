@@ -170,7 +170,7 @@ GroupLowering lower_group(const Program& p, const std::vector<int>& g, const kf_
           A = std::max(A, -L.delay[b]);
     r.A = A;
     r.B = B;
-    r.slots = (A - B + 1) + U * (S - 1);
+    r.slots = (A - B + 1) + U * S - 1;   // planes in use [t+B, t+U-1+A] plus U*(S-1) prefetched
     finish_ring(r);
     L.rings.push_back(r);
   }

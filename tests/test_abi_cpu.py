@@ -117,8 +117,8 @@ def test_search_equals_brute_force(seed):
 
 def test_resource_limits_V7_V8():
     desc = P.tiny()
-    tk = kf.Target(smem_per_block=26895)
-    to = L.Target(smem_per_block=26895)
+    tk = kf.Target(smem_per_block=30095)
+    to = L.Target(smem_per_block=30095)
     check_program(desc, target=(to, tk))
     assert kf.Program(desc).validate([0, 0, 1], tk)[0] == L.V7_SMEM
     tk = kf.Target(regs_per_thread_max=40)

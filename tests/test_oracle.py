@@ -433,11 +433,11 @@ def test_resource_model_worked_example():
     """V7 model (R20), hand-worked for tiny {K1,K2}, fp32, tile 32x16, S=2 stages, U=2 planes/iteration:
     delays D(K1)=0, D(K2)=1 (K2 reads v at dz=+1).
     u (live-in): box x extent below T 2 -> 4 (16-byte TMA start, R20a), width 32+4+2=38 -> row 40,
-      height 20, A=1-0=1, B=-1-0=-1 -> span 3, slots 3+U(S-1)=5, plane roundup(40*20*4,128)=3200
+      height 20, A=1-0=1, B=-1-0=-1 -> span 3, slots 3+U*S-1=6, plane roundup(40*20*4,128)=3200
     v (in-group): box 34x18 -> row 36, span (1-(-1))-0+1 = 3, slots 3+(U-1)=4,
       plane roundup(36*18*4,128)=2688
-    total = 5*3200 + 4*2688 + 8*2 + 128 = 26896;  with U=1: 4*3200 + 3*2688 + 144 = 21008."""
+    total = 6*3200 + 4*2688 + 8*2 + 128 = 30096;  with U=1: 4*3200 + 3*2688 + 144 = 21008."""
     s = L.schedule(P.tiny(), [0, 1], L.Target())
     assert s["delay"] == {0: 0, 1: 1}
-    assert s["smem"] == 5 * 3200 + 4 * 2688 + 16 + 128 == 26896
+    assert s["smem"] == 6 * 3200 + 4 * 2688 + 16 + 128 == 30096
     assert L.schedule(P.tiny(), [0, 1], L.Target(zunroll=1))["smem"] == 21008
