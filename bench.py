@@ -38,7 +38,7 @@ def workload(name: str):
     from workloads import data, programs
     if name == "weather":
         desc = programs.weather(n=(512, 512, 128))
-        return desc, data.weather_inputs, dict(tile=(32, 16, 0)), "weather-44k31a-512x512x128-fp64 (BASELINE config 3)"
+        return desc, data.weather_inputs, dict(tile=(64, 4, 0)), "weather-44k31a-512x512x128-fp64 (BASELINE config 3)"
     if name == "weather_small":
         desc = programs.weather(n=(128, 128, 64))
         return desc, data.weather_inputs, dict(tile=(32, 16, 0)), "weather-44k31a-128x128x64-fp64"
@@ -377,7 +377,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="kf", choices=["kf", "reference"])
     ap.add_argument("--workload", default="weather")
-    ap.add_argument("--plan", default="best", choices=["best", "unfused", "hand"])
+    ap.add_argument("--plan", default="hand", choices=["best", "unfused", "hand"])
     ap.add_argument("--tile", default=None)
     ap.add_argument("--stages", type=int, default=None)
     ap.add_argument("--threads", type=int, default=None)

@@ -36,12 +36,12 @@ class Target:
     smem_per_block: int = 232448
     regs_per_thread_max: int = 255
     n_sm: int = 148
-    tile: Tuple[int, int, int] = (32, 16, 0)
+    tile: Tuple[int, int, int] = (64, 4, 0)
     stages: int = 2
     threads: int = 256
     max_halo: int = 16
     internal_axes: int = 0          # bitmask of axes split across ranks (treated like periodic by V6)
-    zunroll: int = 2                # planes per stream iteration U (ring depth grows with U, R20)
+    zunroll: int = 1                # planes per stream iteration U (ring depth grows with U, R20)
 
 
 # ---------------------------------------------------------------- plans

@@ -335,12 +335,12 @@ kf_status kf_target_b200(kf_target* out) {
     t.smem_per_block = 232448;
     t.regs_per_thread_max = 255;
     t.n_sm = 148;
-    t.tile[0] = 32; t.tile[1] = 16; t.tile[2] = 0;
+    t.tile[0] = 64; t.tile[1] = 4; t.tile[2] = 0;
     t.stages = 2;
     t.threads = 256;
     t.max_halo = 16;
     t.internal_axes = 0;
-    t.zunroll = 2;
+    t.zunroll = 1;
     *out = t;
   });
 }

@@ -117,12 +117,14 @@ def test_search_equals_brute_force(seed):
 
 def test_resource_limits_V7_V8():
     desc = P.tiny()
-    tk = kf.Target(smem_per_block=30095)
-    to = L.Target(smem_per_block=30095)
+    tk = kf.Target(smem_per_block=30095, tile=(32, 16, 0), zunroll=2)
+    to = L.Target(smem_per_block=30095, tile=(32, 16, 0), zunroll=2)
     check_program(desc, target=(to, tk))
     assert kf.Program(desc).validate([0, 0, 1], tk)[0] == L.V7_SMEM
-    tk = kf.Target(regs_per_thread_max=40)
-    to = L.Target(regs_per_thread_max=40)
+    for zu in (1, 3):
+        check_program(desc, target=(L.Target(zunroll=zu, tile=(16, 8, 0)), kf.Target(zunroll=zu, tile=(16, 8, 0))))
+    tk = kf.Target(regs_per_thread_max=40, zunroll=2)
+    to = L.Target(regs_per_thread_max=40, zunroll=2)
     check_program(desc, target=(to, tk))
 
 

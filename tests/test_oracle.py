@@ -437,7 +437,7 @@ def test_resource_model_worked_example():
     v (in-group): box 34x18 -> row 36, span (1-(-1))-0+1 = 3, slots 3+(U-1)=4,
       plane roundup(36*18*4,128)=2688
     total = 6*3200 + 4*2688 + 8*2 + 128 = 30096;  with U=1: 4*3200 + 3*2688 + 144 = 21008."""
-    s = L.schedule(P.tiny(), [0, 1], L.Target())
+    s = L.schedule(P.tiny(), [0, 1], L.Target(tile=(32, 16, 0), zunroll=2))
     assert s["delay"] == {0: 0, 1: 1}
     assert s["smem"] == 6 * 3200 + 4 * 2688 + 16 + 128 == 30096
-    assert L.schedule(P.tiny(), [0, 1], L.Target(zunroll=1))["smem"] == 21008
+    assert L.schedule(P.tiny(), [0, 1], L.Target(tile=(32, 16, 0), zunroll=1))["smem"] == 21008
