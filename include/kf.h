@@ -236,6 +236,11 @@ typedef struct kf_exec kf_exec;
  * per group and JIT-compiles it with NVRTC for sm_100a (--fmad=false, IEEE div/sqrt).
  * Needs a CUDA device (current device of the calling thread). */
 kf_status kf_exec_create(kf_program* prog, const int32_t* plan, const kf_target* target, kf_exec** out);
+/* Same with one launch configuration per fused group: targets[n_targets], n_targets = 1 (all
+ * groups) or m (canonical group order).  Legality V6-V8 is checked per group with its own
+ * target (tile, stages, zunroll, limits) -- e.g. the result of per-group autotuning. */
+kf_status kf_exec_create_ex(kf_program* prog, const int32_t* plan, const kf_target* targets, int32_t n_targets,
+                            kf_exec** out);
 void kf_exec_destroy(kf_exec* ex);
 /* Bytes of caller-provided device scratch: one buffer per renamed array version. */
 kf_status kf_exec_scratch_bytes(const kf_exec* ex, uint64_t* bytes);

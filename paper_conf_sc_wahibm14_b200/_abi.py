@@ -119,6 +119,7 @@ SIGNATURES = {
     "kf_plan_search": (C.c_int, [P, C.POINTER(kf_target), C.c_int32, C.c_uint64, I32P, U64P]),
     "kf_plan_count_legal": (C.c_int, [P, C.POINTER(kf_target), U64P]),
     "kf_exec_create": (C.c_int, [P, I32P, C.POINTER(kf_target), C.POINTER(P)]),
+    "kf_exec_create_ex": (C.c_int, [P, I32P, C.POINTER(kf_target), C.c_int32, C.POINTER(P)]),
     "kf_exec_destroy": (None, [P]),
     "kf_exec_scratch_bytes": (C.c_int, [P, U64P]),
     "kf_exec_run": (C.c_int, [P, C.POINTER(P), P, C.c_uint64, C.c_int64, C.POINTER(C.c_double), P]),

@@ -204,11 +204,16 @@ class Program:
 class Exec:
     """kf_exec: a validated, lowered and JIT-compiled plan (one sm_100a kernel per group)."""
 
-    def __init__(self, program: Program, plan: Sequence[int], target: Optional[Target] = None):
+    def __init__(self, program: Program, plan: Sequence[int], target: Optional[Target] = None,
+                 group_targets: Optional[Sequence[Target]] = None):
         self.program = program
         self.target = target or Target()
         h = C.c_void_p()
-        check(lib().kf_exec_create(program.h, _i32(plan), C.byref(self.target.c), C.byref(h)))
+        if group_targets:
+            arr = (kf_target * len(group_targets))(*[t.c for t in group_targets])
+            check(lib().kf_exec_create_ex(program.h, _i32(plan), arr, len(group_targets), C.byref(h)))
+        else:
+            check(lib().kf_exec_create(program.h, _i32(plan), C.byref(self.target.c), C.byref(h)))
         self.h = h
         self.plan = list(plan)
 

@@ -134,6 +134,9 @@ GroupLowering lower_group(const Program& p, const std::vector<int>& g, const kf_
 // Validation; returns code (0 ok) and fills why.
 int validate_plan(const Program& p, const Plan& pl, const kf_target& t, kf_violation* why,
                   std::vector<GroupLowering>* lowered = nullptr);
+// Same with one launch configuration per group (targets.size() == pl.m).
+int validate_plan_groups(const Program& p, const Plan& pl, const std::vector<kf_target>& targets, kf_violation* why,
+                         std::vector<GroupLowering>* lowered = nullptr);
 std::vector<int> quotient_order(const Program& p, const Plan& pl);   // empty if cyclic
 int check_kinship(const Program& p, const std::vector<int>& g, int gi, kf_violation* why);
 int check_convex(const Program& p, const std::vector<int>& g, int gi, kf_violation* why);

@@ -348,8 +348,8 @@ bool quotient_acyclic(const Program& p, const std::vector<int>& label, int m, in
   return true;
 }
 
-int validate_plan(const Program& p, const Plan& pl, const kf_target& t, kf_violation* why,
-                  std::vector<GroupLowering>* lowered) {
+int validate_plan_groups(const Program& p, const Plan& pl, const std::vector<kf_target>& T, kf_violation* why,
+                         std::vector<GroupLowering>* lowered) {
   if (why) *why = kf_violation{KF_V_OK, -1, -1, -1, -1};
   int c;
   for (int gi = 0; gi < pl.m; gi++)
@@ -362,23 +362,28 @@ int validate_plan(const Program& p, const Plan& pl, const kf_target& t, kf_viola
     return KF_V_CYCLE;
   }
   std::vector<GroupLowering> Ls;
-  for (int gi = 0; gi < pl.m; gi++) Ls.push_back(lower_group(p, pl.groups[gi], t));
+  for (int gi = 0; gi < pl.m; gi++) Ls.push_back(lower_group(p, pl.groups[gi], T[gi]));
   for (int gi = 0; gi < pl.m; gi++)
     if ((c = check_hazard(p, pl.groups[gi], Ls[gi], gi, why))) return c;
   for (int gi = 0; gi < pl.m; gi++)
-    if ((c = check_halo(p, Ls[gi], t, gi, why))) return c;
+    if ((c = check_halo(p, Ls[gi], T[gi], gi, why))) return c;
   for (int gi = 0; gi < pl.m; gi++)
-    if (Ls[gi].smem > t.smem_per_block) {
+    if (Ls[gi].smem > T[gi].smem_per_block) {
       if (why) *why = kf_violation{KF_V_SMEM, gi, -1, -1, -1};
       return KF_V_SMEM;
     }
   for (int gi = 0; gi < pl.m; gi++)
-    if (Ls[gi].regs > t.regs_per_thread_max) {
+    if (Ls[gi].regs > T[gi].regs_per_thread_max) {
       if (why) *why = kf_violation{KF_V_REGS, gi, -1, -1, -1};
       return KF_V_REGS;
     }
   if (lowered) *lowered = std::move(Ls);
   return KF_V_OK;
+}
+
+int validate_plan(const Program& p, const Plan& pl, const kf_target& t, kf_violation* why,
+                  std::vector<GroupLowering>* lowered) {
+  return validate_plan_groups(p, pl, std::vector<kf_target>(pl.m, t), why, lowered);
 }
 
 uint64_t group_bytes(const Program& p, const std::vector<int>& g, uint64_t* rd, uint64_t* wr) {

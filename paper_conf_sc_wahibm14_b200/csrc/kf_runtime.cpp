@@ -468,20 +468,28 @@ static void exec_run(kf_exec* E, void* const* arrays, void* scratch, uint64_t sc
 
 extern "C" {
 
-kf_status kf_exec_create(kf_program* prog, const int32_t* plan, const kf_target* target, kf_exec** out) {
+kf_status kf_exec_create_ex(kf_program* prog, const int32_t* plan, const kf_target* targets, int32_t n_targets,
+                            kf_exec** out) {
   KF_TRY({
-    if (!prog || !plan || !out) fail(KF_E_ARG, "null argument");
-    check_target(target);
+    if (!prog || !plan || !out || !targets || n_targets < 1) fail(KF_E_ARG, "null argument");
     const Program& p = prog->p;
     for (int k = 0; k < p.nk; k++)
       if (plan[k] < 0) fail(KF_E_ILLEGAL_PLAN, "V1 PARTITION: kernel " + std::to_string(k) + " has no group");
     auto E = std::make_unique<kf_exec>();
     E->prog = prog;
-    E->t = *target;
     E->plan = make_plan(p, plan);
+    if (n_targets != 1 && n_targets != E->plan.m)
+      fail(KF_E_ARG, "n_targets must be 1 or the number of groups (" + std::to_string(E->plan.m) + ")");
+    std::vector<kf_target> T;
+    for (int gi = 0; gi < E->plan.m; gi++) {
+      const kf_target& t = targets[n_targets == 1 ? 0 : gi];
+      check_target(&t);
+      T.push_back(t);
+    }
+    E->t = T[0];
     kf_violation why{};
     std::vector<GroupLowering> Ls;
-    int code = validate_plan(p, E->plan, *target, &why, &Ls);
+    int code = validate_plan_groups(p, E->plan, T, &why, &Ls);
     if (code != KF_V_OK)
       fail(KF_E_ILLEGAL_PLAN, "plan violates constraint V" + std::to_string(code) + " in group " + std::to_string(why.group));
     E->order = quotient_order(p, E->plan);
@@ -498,13 +506,14 @@ kf_status kf_exec_create(kf_program* prog, const int32_t* plan, const kf_target*
     E->array_bytes = uint64_t(p.layout.elems) * p.es;
     E->array_bytes = (E->array_bytes + 255) / 256 * 256;
     E->scratch_bytes = E->array_bytes * E->scratch_vers.size();
-    const int TZ = target->tile[2] > 0 ? std::min<int64_t>(target->tile[2], p.n[2]) : int(p.n[2]);
-    int64_t units = ((p.n[0] + target->tile[0] - 1) / target->tile[0]) * ((p.n[1] + target->tile[1] - 1) / target->tile[1]) *
-                    ((p.n[2] + TZ - 1) / TZ);
-    if (units > 2147483647) fail(KF_E_UNSUPPORTED, "grid too large");
     E->G.resize(E->plan.m);
     for (int gi = 0; gi < E->plan.m; gi++) {
       GroupExec& g = E->G[gi];
+      const kf_target& t = T[gi];
+      const int TZ = t.tile[2] > 0 ? std::min<int64_t>(t.tile[2], p.n[2]) : int(p.n[2]);
+      int64_t units = ((p.n[0] + t.tile[0] - 1) / t.tile[0]) * ((p.n[1] + t.tile[1] - 1) / t.tile[1]) *
+                      ((p.n[2] + TZ - 1) / TZ);
+      if (units > 2147483647) fail(KF_E_UNSUPPORTED, "grid too large");
       g.gid = gi;
       g.L = std::move(Ls[gi]);
       g.cg = generate_group_kernel(p, g.L, gi);
@@ -521,6 +530,10 @@ kf_status kf_exec_create(kf_program* prog, const int32_t* plan, const kf_target*
     build_schedule(E.get());
     *out = E.release();
   });
+}
+
+kf_status kf_exec_create(kf_program* prog, const int32_t* plan, const kf_target* target, kf_exec** out) {
+  return kf_exec_create_ex(prog, plan, target, 1, out);
 }
 
 void kf_exec_destroy(kf_exec* ex) {

@@ -133,3 +133,23 @@ def test_run_host_path():
     got = {nm: prog.from_device_layout(t.numpy()) for (nm, _), t in zip(desc.arrays, host)}
     assert compare(desc, got, interp.run(desc, inputs, 3)) == []
     assert h2d > 0 and d2h > 0
+
+
+def test_per_group_launch_configs():
+    """kf_exec_create_ex: every group with its own tile / stages / zunroll, bit-exact."""
+    from workloads.programs import weather_hand_plan
+    desc = P.weather(n=(40, 36, 10))
+    inputs = D.inputs_for(desc, 7)
+    ref = interp.run(desc, inputs, 2)
+    plan = weather_hand_plan(desc)
+    m = max(plan) + 1
+    cfgs = [((64, 4, 0), 2, 1), ((32, 8, 0), 2, 2), ((16, 8, 3), 3, 1), ((32, 4, 0), 2, 3)]
+    tg = [kf.Target(tile=cfgs[g % 4][0], stages=cfgs[g % 4][1], zunroll=cfgs[g % 4][2]) for g in range(m)]
+    prog = kf.Program(desc)
+    ex = kf.Exec(prog, plan, group_targets=tg)
+    dev = kf.device_arrays(prog, inputs)
+    sb = ex.scratch_bytes()
+    scratch = torch.empty(sb, dtype=torch.uint8, device="cuda") if sb else None
+    ex.run(dev, scratch, 2)
+    torch.cuda.synchronize()
+    assert compare(desc, kf.host_arrays(prog, dev), ref) == []
