@@ -209,7 +209,9 @@ GroupLowering lower_group(const Program& p, const std::vector<int>& g, const kf_
       maxr = std::max(maxr, (TX + e.elo[0] + e.ehi[0]) * (TY + e.elo[1] + e.ehi[1]));
     }
     int nt = (maxr + 31) / 32 * 32;
-    L.threads = (nt > t.threads && nt <= 512) ? nt : t.threads;
+    // only when the tile itself has at most one point per thread; otherwise the unrolled
+    // rounds of the fast path absorb the halo (critical path P+1 rounds instead of P)
+    L.threads = (t.tile[0] * t.tile[1] <= t.threads && nt > t.threads && nt <= 512) ? nt : t.threads;
   }
   int depth = 1;
   for (int k : g) depth = std::max(depth, p.kernels[k].depth);

@@ -93,7 +93,7 @@ def test_weather_small_fp64_plans():
     desc = P.weather(n=(48, 40, 12))
     inputs = D.inputs_for(desc, 3)
     ref = interp.run(desc, inputs, 2)
-    plan_g, _ = kf.Program(desc).search(kf.SEARCH_GREEDY)
+    plan_g, _ = kf.Program(desc).search(kf.SEARCH_GREEDY, kf.Target(tile=(32, 8, 0), zunroll=2))
     for plan in (list(range(44)), weather_hand_plan(desc), plan_g):
         for zu in (1, 2):
             got, _ = run_kf(desc, plan, inputs, 2, kf.Target(tile=(32, 8, 0), zunroll=zu))
