@@ -42,6 +42,7 @@ class Target:
     max_halo: int = 16
     internal_axes: int = 0          # bitmask of axes split across ranks (treated like periodic by V6)
     zunroll: int = 1                # planes per stream iteration U (ring depth grows with U, R20)
+    pblock: Tuple[int, int] = (1, 1)  # points per thread in x, y (register blocking)
 
 
 # ---------------------------------------------------------------- plans
@@ -227,7 +228,19 @@ def schedule(prog: Program, grp: List[int], target: Target):
         smem += r[5] * plane
     smem += 8 * S + 128
     depth = max([rpn_depth(s.rpn) for k in grp for s in prog.kernels[k].stmts] + [1])
-    regs = 32 + 2 * (es // 4) * (depth + 3)
+    # threads per CTA: cover the largest extended region in one pass when the tile has at most one
+    # point per thread (<= 512); points per thread P = pblock x zunroll x rounds (capped at 8)
+    regions = [((TX + ext[k][0][0] + ext[k][1][0]), (TY + ext[k][0][1] + ext[k][1][1])) for k in alive]
+    maxr = max([w * h for w, h in regions] + [0])
+    nt = _roundup(maxr, 32)
+    threads = nt if (TX * TY <= target.threads and target.threads < nt <= 512) else target.threads
+    rounds = 1
+    for w, h in regions:
+        bx, by = min(target.pblock[0], w), min(target.pblock[1], h)
+        nb = (-(-w // bx)) * (-(-h // by))
+        rounds = max(rounds, -(-nb // threads))
+    P = min(8, target.pblock[0] * target.pblock[1] * target.zunroll * rounds)
+    regs = 32 + 2 * (es // 4) * (depth + 3) * P
     return dict(ext=ext, pts=pts, delay=D, res=res, smem=smem, regs=regs, alive=alive)
 
 

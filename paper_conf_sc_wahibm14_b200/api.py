@@ -26,16 +26,17 @@ class Target:
         t = kf_target()
         check(lib().kf_target_b200(C.byref(t)))
         for k, v in kw.items():
-            if k == "tile":
+            if k in ("tile", "pblock"):
+                arr = getattr(t, k)
                 for i, x in enumerate(v):
-                    t.tile[i] = int(x)
+                    arr[i] = int(x)
             else:
                 setattr(t, k, v)
         self.c = t
 
     def __getattr__(self, k):
-        if k == "tile":
-            return tuple(self.c.tile)
+        if k in ("tile", "pblock"):
+            return tuple(getattr(self.__dict__["c"], k))
         return getattr(self.__dict__["c"], k)
 
 

@@ -125,6 +125,7 @@ struct GroupLowering {
   int mbar_off = 0;
   int tile[3];
   int stages = 2, threads = 256, zunroll = 1;
+  int pblock[2] = {1, 1};   // points per thread in x, y (register blocking in the fast path)
   int ring_of(const Ver& v) const;        // index in rings or -1
 };
 

@@ -75,6 +75,8 @@ GroupLowering lower_group(const Program& p, const std::vector<int>& g, const kf_
   L.stages = t.stages;
   L.threads = t.threads;
   L.zunroll = t.zunroll;
+  L.pblock[0] = t.pblock[0];
+  L.pblock[1] = t.pblock[1];
   L.live_in = group_live_in(p, g);
   L.live_out = group_live_out(p, g);
   L.live_out_set = std::set<Ver>(L.live_out.begin(), L.live_out.end());
@@ -216,7 +218,17 @@ GroupLowering lower_group(const Program& p, const std::vector<int>& g, const kf_
   int depth = 1;
   for (int k : g) depth = std::max(depth, p.kernels[k].depth);
   L.depth = depth;
-  L.regs = 32 + 2 * (es / 4) * (depth + 3);
+  // points computed concurrently per thread in the fast path: blocks x planes x rounds (R20)
+  int rounds = 1;
+  for (int k : alive) {
+    const Ext& e = L.ext[k];
+    const int WX = TX + e.elo[0] + e.ehi[0], WY = TY + e.elo[1] + e.ehi[1];
+    const int bx = std::min(t.pblock[0], WX), by = std::min(t.pblock[1], WY);
+    const int nb = ((WX + bx - 1) / bx) * ((WY + by - 1) / by);
+    rounds = std::max(rounds, (nb + L.threads - 1) / L.threads);
+  }
+  const int P = std::min(8, t.pblock[0] * t.pblock[1] * U * rounds);
+  L.regs = 32 + 2 * (es / 4) * (depth + 3) * P;
   return L;
 }
 
@@ -405,6 +417,8 @@ void check_target(const kf_target* t) {
   if (t->tile[0] % 4) fail(KF_E_ARG, "tile TX must be a multiple of 4 (16-byte aligned TMA boxes)");
   if (t->stages < 2 || t->stages > 8) fail(KF_E_ARG, "stages must be in [2, 8]");
   if (t->zunroll < 1 || t->zunroll > 4) fail(KF_E_ARG, "zunroll must be in [1, 4]");
+  if (t->pblock[0] < 1 || t->pblock[0] > 4 || t->pblock[1] < 1 || t->pblock[1] > 4)
+    fail(KF_E_ARG, "pblock must be in [1, 4] x [1, 4]");
   if (t->threads < 32 || t->threads > 1024 || t->threads % 32) fail(KF_E_ARG, "threads must be a multiple of 32 in [32,1024]");
   if (!(t->hbm_bytes_per_s > 0)) fail(KF_E_ARG, "hbm_bytes_per_s must be > 0");
 }

@@ -341,6 +341,8 @@ kf_status kf_target_b200(kf_target* out) {
     t.max_halo = 16;
     t.internal_axes = 0;
     t.zunroll = 1;
+    t.pblock[0] = 1;
+    t.pblock[1] = 1;
     *out = t;
   });
 }

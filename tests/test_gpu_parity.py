@@ -82,8 +82,9 @@ def test_random_programs_random_legal_plans(seed):
     pick = [legal[i] for i in sorted(set(rng.integers(0, len(legal), size=4).tolist()))]
     tile = [(32, 16, 0), (16, 16, 0), (8, 4, 6), (32, 8, 11)][seed % 4]
     zu = [1, 2, 3][seed % 3]
+    pb = [(1, 1), (2, 1), (2, 2), (1, 3)][seed % 4]
     for plan in pick:
-        got, _ = run_kf(desc, plan, inputs, nsteps, kf.Target(tile=tile, zunroll=zu))
+        got, _ = run_kf(desc, plan, inputs, nsteps, kf.Target(tile=tile, zunroll=zu, pblock=pb, threads=64))
         assert compare(desc, got, ref) == [], (plan, tile)
 
 
@@ -143,8 +144,10 @@ def test_per_group_launch_configs():
     ref = interp.run(desc, inputs, 2)
     plan = weather_hand_plan(desc)
     m = max(plan) + 1
-    cfgs = [((64, 4, 0), 2, 1), ((32, 8, 0), 2, 2), ((16, 8, 3), 3, 1), ((32, 4, 0), 2, 3)]
-    tg = [kf.Target(tile=cfgs[g % 4][0], stages=cfgs[g % 4][1], zunroll=cfgs[g % 4][2]) for g in range(m)]
+    cfgs = [((64, 4, 0), 2, 1, (1, 1), 256), ((32, 8, 0), 2, 2, (2, 2), 128), ((16, 8, 3), 3, 1, (1, 2), 64),
+            ((32, 4, 0), 2, 3, (2, 1), 64), ((64, 8, 0), 2, 1, (2, 2), 128)]
+    tg = [kf.Target(tile=cfgs[g % 5][0], stages=cfgs[g % 5][1], zunroll=cfgs[g % 5][2], pblock=cfgs[g % 5][3],
+                    threads=cfgs[g % 5][4]) for g in range(m)]
     prog = kf.Program(desc)
     ex = kf.Exec(prog, plan, group_targets=tg)
     dev = kf.device_arrays(prog, inputs)

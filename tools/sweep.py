@@ -16,8 +16,9 @@ def main():
     out = []
     for cfg in configs:
         tile, stages, threads = cfg[:3]
-        zu = cfg[3] if len(cfg) > 3 else 2
-        tgt = kf.Target(tile=tile, stages=stages, threads=threads, zunroll=zu)
+        zu = cfg[3] if len(cfg) > 3 else 1
+        pb = cfg[4] if len(cfg) > 4 else [1, 1]
+        tgt = kf.Target(tile=tile, stages=stages, threads=threads, zunroll=zu, pblock=pb)
         if plan_kind == "hand":
             plan = P.weather_hand_plan(desc)
         elif plan_kind == "unfused":
@@ -42,7 +43,7 @@ def main():
         ms = e0.elapsed_time(e1) / 10
         gms, _ = ex.group_times()
         info = ex.info()
-        r = {"tile": tile, "stages": stages, "threads": threads, "zunroll": zu, "ms_per_step": ms,
+        r = {"tile": tile, "stages": stages, "threads": threads, "zunroll": zu, "pblock": pb, "ms_per_step": ms,
              "TBps": info.compulsory_bytes_per_step / ms / 1e9,
              "groups": [(ex.group_info(g).name.decode(), round(gms[g] / 10, 4),
                          round(ex.group_info(g).bytes_per_launch / (gms[g] / 10) / 1e9, 2),
