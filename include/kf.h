@@ -205,7 +205,8 @@ typedef struct {
   uint64_t halo_bytes_est;       /* tile-halo re-reads over the interior (not compulsory)  */
   uint32_t smem_bytes, regs_est;
   int32_t n_kernels, unprofitable;
-  double t_s;
+  double t_s;                    /* codeless bound: compulsory bytes / hbm_bytes_per_s            */
+  double t_model_s;              /* resource-aware projection (R22): HBM + issue time of regions  */
 } kf_group_proj;
 kf_status kf_project(const kf_program* prog, const int32_t* plan, const kf_target* target,
                      kf_group_proj* per_group, int32_t cap, int32_t* m,
@@ -222,10 +223,13 @@ kf_status kf_group_schedule(const kf_program* prog, const int32_t* plan, const k
 typedef enum {
   KF_SEARCH_BRUTE = 0,   /* all restricted-growth strings with pruning (n <= 14)           */
   KF_SEARCH_GREEDY = 1,  /* agglomerative merging of groups by largest byte saving          */
-  KF_SEARCH_AUTO = 2     /* brute if n <= 10 else greedy                                    */
+  KF_SEARCH_AUTO = 2,    /* brute if n <= 10 else greedy                                    */
+  KF_SEARCH_GREEDY_TIME = 3,  /* greedy merging on the resource-aware projected time (R22)    */
+  KF_SEARCH_BRUTE_TIME = 4    /* brute force on the resource-aware projected time (n <= 14)    */
 } kf_search_method;
-/* Minimises total compulsory bytes over legal plans; ties -> lexicographically smallest
- * canonical labels (R17).  plan_out: int32_t[n] canonical.  bytes_out may be NULL. */
+/* Minimises total compulsory bytes (or, for the *_TIME methods, total projected time) over
+ * legal plans; ties -> lexicographically smallest canonical labels (R17).  plan_out:
+ * int32_t[n] canonical.  bytes_out (compulsory bytes of the result) may be NULL. */
 kf_status kf_plan_search(const kf_program* prog, const kf_target* target, int32_t method,
                          uint64_t seed, int32_t* plan_out, uint64_t* bytes_out);
 /* Number of legal partitions (brute force; n <= 14). */

@@ -5,5 +5,6 @@ projection, plan search, NVRTC-JIT'd sm_100a group kernels and the step runtime.
 This package is only the ctypes binding; it never computes anything itself.
 """
 from ._abi import KfError, lib  # noqa: F401
-from .api import (SEARCH_AUTO, SEARCH_BRUTE, SEARCH_GREEDY, Exec, Program, Target,  # noqa: F401
+from .api import (SEARCH_AUTO, SEARCH_BRUTE, SEARCH_BRUTE_TIME, SEARCH_GREEDY, SEARCH_GREEDY_TIME,  # noqa: F401
+                  Exec, Program, Target,
                   device_arrays, flush_l2, host_arrays)

@@ -75,7 +75,7 @@ class kf_violation(C.Structure):
 class kf_group_proj(C.Structure):
     _fields_ = [("bytes_read", C.c_uint64), ("bytes_written", C.c_uint64), ("halo_bytes_est", C.c_uint64),
                 ("smem_bytes", C.c_uint32), ("regs_est", C.c_uint32), ("n_kernels", C.c_int32),
-                ("unprofitable", C.c_int32), ("t_s", C.c_double)]
+                ("unprofitable", C.c_int32), ("t_s", C.c_double), ("t_model_s", C.c_double)]
 
 
 class kf_kernel_sched(C.Structure):

@@ -146,6 +146,9 @@ int check_halo(const Program& p, const GroupLowering& L, const kf_target& t, int
 bool quotient_acyclic(const Program& p, const std::vector<int>& label, int m, int* first_bad);
 void check_target(const kf_target* t);
 uint64_t group_bytes(const Program& p, const std::vector<int>& g, uint64_t* rd, uint64_t* wr);
+// Resource-aware projected time of one fused group (NEXT-2 direction, R22): HBM time of the
+// compulsory bytes at the achievable copy rate, plus issue time of the recomputed regions.
+double model_time(const Program& p, const GroupLowering& L, const kf_target& t, uint64_t bytes);
 
 // ---------------------------------------------------------------- codegen
 struct Codegen {

@@ -409,6 +409,31 @@ uint64_t group_bytes(const Program& p, const std::vector<int>& g, uint64_t* rd, 
   return r + w;
 }
 
+double model_time(const Program& p, const GroupLowering& L, const kf_target& t, uint64_t bytes) {
+  // Calibrated on B200 (profiles/round1_summary.md): ~17 issue slots of fixed cost per point of
+  // an extended region plus ~1.5 per RPN node / store; ~2.5e13 thread-instructions/s sustained;
+  // compulsory bytes at 79% of nominal HBM (the measured copy rate); memory and issue overlap
+  // by half the shorter of the two.  A model, not a measurement (reported beside measured times).
+  const double T = double(L.tile[0]) * L.tile[1];
+  double work = 0.0;
+  for (int k : L.kernels) {
+    const Ext& e = L.ext.at(k);
+    if (!e.alive) continue;
+    const double R = double(L.tile[0] + e.elo[0] + e.ehi[0]) * (L.tile[1] + e.elo[1] + e.ehi[1]);
+    int ops = 0;
+    for (auto& st : p.kernels[k].stmts) ops += int(st.rpn.size()) + 1;
+    work += (R / T) * (17.0 + 1.5 * ops);
+  }
+  // issue efficiency falls with the warps an SM can hold (SMEM-limited CTAs x warps per CTA):
+  // full rate from 32 resident warps, proportionally less below (latency no longer hidden)
+  const int ctas = std::max(1, std::min(2048 / std::max(32, L.threads), 233472 / std::max(1, L.smem + 1024)));
+  const double warps = std::min(64.0, double(ctas) * (L.threads / 32));
+  const double eff = std::min(1.0, warps / 32.0);
+  const double t_comp = double(p.npts) * work / (2.5e13 * eff);
+  const double t_mem = double(bytes) / (0.79 * t.hbm_bytes_per_s);
+  return t_mem + t_comp - 0.5 * std::min(t_mem, t_comp) + 5e-6;
+}
+
 void check_target(const kf_target* t) {
   if (!t) fail(KF_E_ARG, "null target");
   if (t->tile[0] < 1 || t->tile[1] < 1 || t->tile[2] < 0 || t->tile[0] > 224 || t->tile[1] > 224)
@@ -507,6 +532,7 @@ kf_status kf_project(const kf_program* prog, const int32_t* plan, const kf_targe
         r.unprofitable = (r.bytes_read + r.bytes_written) >= alone;
       }
       r.t_s = double(r.bytes_read + r.bytes_written) / target->hbm_bytes_per_s;
+      r.t_model_s = model_time(p, L, *target, r.bytes_read + r.bytes_written);
       tot += r.bytes_read + r.bytes_written;
       tt += r.t_s;
       res.push_back(r);

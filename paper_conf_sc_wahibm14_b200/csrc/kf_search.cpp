@@ -20,6 +20,7 @@ namespace kf {
 struct GroupVerdict {
   bool ok;
   uint64_t bytes;
+  double t_model;
 };
 
 class Evaluator {
@@ -30,7 +31,7 @@ class Evaluator {
     std::string key(reinterpret_cast<const char*>(g.data()), g.size() * sizeof(int));
     auto it = cache_.find(key);
     if (it != cache_.end()) return it->second;
-    GroupVerdict v{true, group_bytes(p_, g, nullptr, nullptr)};
+    GroupVerdict v{true, group_bytes(p_, g, nullptr, nullptr), 0.0};
     if (check_kinship(p_, g, 0, nullptr) || check_convex(p_, g, 0, nullptr)) {
       v.ok = false;
     } else {
@@ -38,21 +39,26 @@ class Evaluator {
       if (check_hazard(p_, g, L, 0, nullptr) || check_halo(p_, L, t_, 0, nullptr) || L.smem > t_.smem_per_block ||
           L.regs > t_.regs_per_thread_max)
         v.ok = false;
+      else
+        v.t_model = model_time(p_, L, t_, v.bytes);
     }
     return cache_.emplace(key, v).first->second;
   }
   // Full legality of a canonical labelling.
-  bool legal(const std::vector<int>& label, int m, uint64_t* bytes) {
+  bool legal(const std::vector<int>& label, int m, uint64_t* bytes, double* tmodel = nullptr) {
     std::vector<std::vector<int>> gs(m);
     for (int k = 0; k < int(label.size()); k++) gs[label[k]].push_back(k);
     uint64_t tot = 0;
+    double tt = 0.0;
     for (auto& g : gs) {
       const GroupVerdict& v = eval(g);
       if (!v.ok) return false;
       tot += v.bytes;
+      tt += v.t_model;
     }
     if (!quotient_acyclic(p_, label, m, nullptr)) return false;
     if (bytes) *bytes = tot;
+    if (tmodel) *tmodel = tt;
     return true;
   }
 
@@ -106,16 +112,24 @@ static std::vector<int> canon(const std::vector<int>& lab, int* m) {
   return out;
 }
 
-static std::vector<int> greedy(const Program& p, Evaluator& ev, uint64_t* best_bytes) {
+static std::vector<int> greedy(const Program& p, Evaluator& ev, uint64_t* best_bytes, bool by_time) {
   std::vector<int> label(p.nk);
   for (int k = 0; k < p.nk; k++) label[k] = k;
   int m = p.nk;
-  uint64_t cur = 0;
-  ev.legal(label, m, &cur);
+  // objective: compulsory bytes, or projected time (scaled to an integer-like double)
+  auto cost = [&](const std::vector<int>& lab, int mm, double* c) {
+    uint64_t b = 0;
+    double t = 0.0;
+    if (!ev.legal(lab, mm, &b, &t)) return false;
+    *c = by_time ? t : double(b);
+    return true;
+  };
+  double cur = 0.0;
+  cost(label, m, &cur);
   for (;;) {
     std::vector<std::vector<int>> gs(m);
     for (int k = 0; k < p.nk; k++) gs[label[k]].push_back(k);
-    uint64_t best = cur;
+    double best = cur;
     std::vector<int> best_lab;
     for (int gi = 0; gi < m; gi++)
       for (int gj = gi + 1; gj < m; gj++) {
@@ -148,8 +162,8 @@ static std::vector<int> greedy(const Program& p, Evaluator& ev, uint64_t* best_b
           if (merged.count(lab[k])) lab[k] = tgt;
         int mm = 0;
         lab = canon(lab, &mm);
-        uint64_t b = 0;
-        if (!ev.legal(lab, mm, &b)) continue;
+        double b = 0.0;
+        if (!cost(lab, mm, &b)) continue;
         if (b < cur && (best_lab.empty() || b < best || (b == best && lab < best_lab))) {
           best = b;
           best_lab = lab;
@@ -161,7 +175,12 @@ static std::vector<int> greedy(const Program& p, Evaluator& ev, uint64_t* best_b
     m = 0;
     label = canon(label, &m);
   }
-  if (best_bytes) *best_bytes = cur;
+  if (best_bytes) {
+    int mm = *std::max_element(label.begin(), label.end()) + 1;
+    uint64_t b = 0;
+    ev.legal(label, mm, &b);
+    *best_bytes = b;
+  }
   return label;
 }
 
@@ -182,17 +201,21 @@ kf_status kf_plan_search(const kf_program* prog, const kf_target* target, int32_
     if (method == KF_SEARCH_AUTO) method = p.nk <= 10 ? KF_SEARCH_BRUTE : KF_SEARCH_GREEDY;
     std::vector<int> best;
     uint64_t best_b = 0;
-    if (method == KF_SEARCH_BRUTE) {
+    if (method == KF_SEARCH_BRUTE || method == KF_SEARCH_BRUTE_TIME) {
       if (p.nk > 14) fail(KF_E_UNSUPPORTED, "brute-force search limited to 14 kernels");
       bool have = false;
+      double best_t = 0.0;
+      const bool by_time = method == KF_SEARCH_BRUTE_TIME;
       enumerate(p, [&](const std::vector<int>& lab, int m) {
         uint64_t b;
-        if (!ev.legal(lab, m, &b)) return;
-        if (!have || b < best_b) { best = lab; best_b = b; have = true; }   // RGS order = lexicographic
+        double t;
+        if (!ev.legal(lab, m, &b, &t)) return;
+        bool better = by_time ? (!have || t < best_t) : (!have || b < best_b);   // RGS order = lexicographic
+        if (better) { best = lab; best_b = b; best_t = t; have = true; }
       });
       if (!have) fail(KF_E_ILLEGAL_PLAN, "no legal plan");   // cannot happen: singletons are legal unless V6-V8 bind
-    } else if (method == KF_SEARCH_GREEDY) {
-      best = greedy(p, ev, &best_b);
+    } else if (method == KF_SEARCH_GREEDY || method == KF_SEARCH_GREEDY_TIME) {
+      best = greedy(p, ev, &best_b, method == KF_SEARCH_GREEDY_TIME);
       int m = 0;
       if (!ev.legal(best, *std::max_element(best.begin(), best.end()) + 1, nullptr))
         fail(KF_E_ILLEGAL_PLAN, "even the unfused plan is illegal under this target");

@@ -8,7 +8,8 @@ from workloads import programs as P, data as D
 def main():
     plan_kind = sys.argv[1] if len(sys.argv) > 1 else "hand"
     configs = json.loads(sys.argv[2]) if len(sys.argv) > 2 else [[[32, 16, 0], 2, 256]]
-    desc = P.weather(n=(512, 512, 128))
+    from workloads.program import PROG_RELAX_ALL, PROG_RELAX_EXPANDABLE
+    desc = P.weather(n=(512, 512, 128), relax=PROG_RELAX_ALL if plan_kind.endswith("_all") else PROG_RELAX_EXPANDABLE)
     prog = kf.Program(desc)
     inputs = D.weather_inputs(desc, 3)
     dev = kf.device_arrays(prog, inputs)
@@ -23,6 +24,8 @@ def main():
             plan = P.weather_hand_plan(desc)
         elif plan_kind == "unfused":
             plan = list(range(44))
+        elif plan_kind.startswith("time"):
+            plan, _ = prog.search(kf.SEARCH_GREEDY_TIME, tgt)
         else:
             plan, _ = prog.search(kf.SEARCH_GREEDY, tgt)
         try:
@@ -43,7 +46,8 @@ def main():
         ms = e0.elapsed_time(e1) / 10
         gms, _ = ex.group_times()
         info = ex.info()
-        r = {"tile": tile, "stages": stages, "threads": threads, "zunroll": zu, "pblock": pb, "ms_per_step": ms,
+        per, _, _ = prog.project(plan, tgt)
+        r = {"plan": plan_kind, "model_ms": sum(g.t_model_s for g in per) * 1e3, "tile": tile, "stages": stages, "threads": threads, "zunroll": zu, "pblock": pb, "ms_per_step": ms,
              "TBps": info.compulsory_bytes_per_step / ms / 1e9,
              "groups": [(ex.group_info(g).name.decode(), round(gms[g] / 10, 4),
                          round(ex.group_info(g).bytes_per_launch / (gms[g] / 10) / 1e9, 2),
