@@ -294,6 +294,27 @@ kf_status kf_exec_group_times(kf_exec* ex, double* ms, int32_t cap, int32_t* n, 
 /* Use a captured CUDA graph for the step loop (default on). */
 kf_status kf_exec_set_graph(kf_exec* ex, int32_t on);
 
+/* ------------------------------------------------------------------ multi-GPU (row a11) */
+/* Domain decomposition over a px x py process grid (x, y split; z whole; part/rank index
+ * iy*px + ix).  Every part runs the same kf_exec plan on its LOCAL sub-domain (the local
+ * program has n = global n / (px, py) and PERIODIC bc on decomposed axes); the periodic
+ * ghost fills of the schedule become halo exchanges with neighbouring parts (x strips, then
+ * y strips incl. x ghosts = corners), so results equal the single-domain run bit for bit.
+ * Transports: loopback -- n_parts == px*py, world == 1: all parts in this process on one
+ * device (strips copied device-to-device; for testing); NCCL -- n_parts == 1,
+ * world == px*py, rank in [0, world): ncclSend/ncclRecv per neighbour over NVLink/NVSwitch,
+ * nccl_id from kf_dist_unique_id() on rank 0, broadcast by the caller (e.g. torch.distributed). */
+typedef struct kf_dist kf_dist;
+kf_status kf_dist_unique_id(uint8_t id[128]);
+kf_status kf_dist_neighbors(int32_t px, int32_t py, int32_t rank, int32_t out[4]);   /* x-, x+, y-, y+ */
+kf_status kf_dist_create(kf_exec* const* parts, int32_t n_parts, int32_t px, int32_t py, int32_t rank, int32_t world,
+                         const uint8_t* nccl_id, kf_dist** out);
+/* arrays: n_parts * n_arrays device pointers (part-major); scratch: n_parts pointers (or NULL
+ * if the plan needs none), each >= kf_exec_scratch_bytes.  Asynchronous on cuda_stream. */
+kf_status kf_dist_run(kf_dist* d, void* const* arrays, void* const* scratch, uint64_t scratch_bytes, int64_t nsteps,
+                      const double* params, void* cuda_stream);
+void kf_dist_destroy(kf_dist* d);
+
 /* ------------------------------------------------------------------ utilities */
 /* Overwrite `bytes` of caller-provided device memory on `cuda_stream` (benchmarks: evict
  * the 126 MB L2 between timed iterations). */

@@ -7,4 +7,5 @@ This package is only the ctypes binding; it never computes anything itself.
 from ._abi import KfError, lib  # noqa: F401
 from .api import (SEARCH_AUTO, SEARCH_BRUTE, SEARCH_BRUTE_TIME, SEARCH_GREEDY, SEARCH_GREEDY_TIME,  # noqa: F401
                   Exec, Program, Target,
-                  device_arrays, flush_l2, host_arrays)
+                  Dist, device_arrays, dist_neighbors, dist_unique_id, flush_l2, gather_domain, host_arrays,
+                  split_domain)

@@ -302,3 +302,77 @@ def device_arrays(program: Program, np_arrays: Dict[str, np.ndarray], device="cu
 
 def host_arrays(program: Program, tensors) -> Dict[str, np.ndarray]:
     return {nm: program.from_device_layout(t.cpu().numpy()) for (nm, _), t in zip(program.desc.arrays, tensors)}
+
+
+class Dist:
+    """kf_dist: a plan run over a px x py domain decomposition (include/kf.h, row a11).
+
+    Loopback (one process, one GPU): Dist(parts=[Exec]*px*py, px, py).
+    NCCL (one process per GPU): Dist([Exec], px, py, rank, world, nccl_id)."""
+
+    def __init__(self, parts: Sequence[Exec], px: int, py: int, rank: int = 0, world: int = 1,
+                 nccl_id: Optional[bytes] = None):
+        self.parts = list(parts)
+        hs = (C.c_void_p * len(parts))(*[e.h for e in parts])
+        idb = (C.c_uint8 * 128)(*nccl_id) if nccl_id is not None else None
+        h = C.c_void_p()
+        check(lib().kf_dist_create(hs, len(parts), px, py, rank, world, idb, C.byref(h)))
+        self.h = h
+
+    def __del__(self):
+        h = getattr(self, "h", None)
+        if h:
+            lib().kf_dist_destroy(h)
+            self.h = None
+
+    def run(self, part_tensors, part_scratch, nsteps: int, params=None, stream=None):
+        import torch
+        stream = stream or torch.cuda.current_stream()
+        ptrs = [t.data_ptr() for ts in part_tensors for t in ts]
+        arr = (C.c_void_p * len(ptrs))(*ptrs)
+        scr = [s.data_ptr() if s is not None else 0 for s in part_scratch]
+        sb = min([s.numel() for s in part_scratch if s is not None] or [0])
+        sarr = (C.c_void_p * len(scr))(*scr)
+        prm = params if params is not None else self.parts[0].program.desc.params
+        pr = (C.c_double * max(1, len(prm)))(*prm)
+        check(lib().kf_dist_run(self.h, arr, sarr, sb, nsteps, pr, C.c_void_p(stream.cuda_stream)))
+
+
+def dist_unique_id() -> bytes:
+    buf = (C.c_uint8 * 128)()
+    check(lib().kf_dist_unique_id(buf))
+    return bytes(buf)
+
+
+def dist_neighbors(px: int, py: int, rank: int):
+    out = (C.c_int32 * 4)()
+    check(lib().kf_dist_neighbors(px, py, rank, out))
+    return list(out)
+
+
+def split_domain(global_desc, arrays: Dict[str, np.ndarray], px: int, py: int):
+    """Cut logical ghosted global arrays into px*py local ones (part-major, iy*px+ix) -- plumbing."""
+    nx, ny, nz = global_desc.n
+    gx, gy, gz = global_desc.ghost
+    assert nx % px == 0 and ny % py == 0, "grid must divide evenly"
+    lx, ly = nx // px, ny // py
+    parts = []
+    for iy in range(py):
+        for ix in range(px):
+            parts.append({nm: np.ascontiguousarray(a[:, iy * ly:iy * ly + ly + 2 * gy, ix * lx:ix * lx + lx + 2 * gx])
+                          for nm, a in arrays.items()})
+    return parts, global_desc.with_(n=(lx, ly, nz))
+
+
+def gather_domain(global_desc, parts: Sequence[Dict[str, np.ndarray]], px: int, py: int, base: Dict[str, np.ndarray]):
+    """Inverse of split_domain for the interiors (ghost cells taken from `base`)."""
+    nx, ny, nz = global_desc.n
+    gx, gy, gz = global_desc.ghost
+    lx, ly = nx // px, ny // py
+    out = {nm: a.copy() for nm, a in base.items()}
+    for r, part in enumerate(parts):
+        ix, iy = r % px, r // px
+        for nm, a in part.items():
+            out[nm][gz:gz + nz, gy + iy * ly:gy + (iy + 1) * ly, gx + ix * lx:gx + (ix + 1) * lx] = \
+                a[gz:gz + nz, gy:gy + ly, gx:gx + lx]
+    return out

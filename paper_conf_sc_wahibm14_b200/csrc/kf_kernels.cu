@@ -76,6 +76,20 @@ __global__ void copy_shell(T* __restrict__ dst, const T* __restrict__ src, Geom 
   }
 }
 
+// Copy a w x h x d box between two buffers (elements; arbitrary pitches): halo strips for
+// domain decomposition (loopback transport) and pack/unpack to contiguous NCCL staging.
+template <typename T>
+__global__ void copy_box(T* __restrict__ dst, long long dpitch, long long dplane, const T* __restrict__ src,
+                         long long spitch, long long splane, int w, int h, int d) {
+  const long long total = (long long)w * h * d;
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
+    const int x = int(i % w);
+    const long long r = i / w;
+    const int y = int(r % h), z = int(r / h);
+    dst[z * dplane + y * dpitch + x] = src[z * splane + y * spitch + x];
+  }
+}
+
 __global__ void flush_kernel(uint4* __restrict__ buf, long long n, unsigned v) {
   for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x)
     buf[i] = make_uint4(v, v + 1, v + 2, v + 3);
@@ -109,6 +123,16 @@ cudaError_t launch_copy_shell(void* dst, const void* src, int es, const Geom& g,
   int nb = blocks_for(n);
   if (es == 4) copy_shell<float><<<nb, 256, 0, s>>>((float*)dst, (const float*)src, g);
   else copy_shell<double><<<nb, 256, 0, s>>>((double*)dst, (const double*)src, g);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_copy_box(void* dst, long long dpitch, long long dplane, const void* src, long long spitch,
+                            long long splane, int w, int h, int d, int es, cudaStream_t s) {
+  long long n = (long long)w * h * d;
+  if (n == 0) return cudaSuccess;
+  int nb = blocks_for(n);
+  if (es == 4) copy_box<float><<<nb, 256, 0, s>>>((float*)dst, dpitch, dplane, (const float*)src, spitch, splane, w, h, d);
+  else copy_box<double><<<nb, 256, 0, s>>>((double*)dst, dpitch, dplane, (const double*)src, spitch, splane, w, h, d);
   return cudaGetLastError();
 }
 

@@ -10,5 +10,7 @@ struct Geom {
 };
 cudaError_t launch_fill(int axis, void* base, int es, const Geom& g, cudaStream_t s);
 cudaError_t launch_copy_shell(void* dst, const void* src, int es, const Geom& g, cudaStream_t s);
+cudaError_t launch_copy_box(void* dst, long long dpitch, long long dplane, const void* src, long long spitch,
+                            long long splane, int w, int h, int d, int es, cudaStream_t s);
 cudaError_t launch_flush(void* buf, long long bytes, unsigned v, cudaStream_t s);
 }  // namespace kf

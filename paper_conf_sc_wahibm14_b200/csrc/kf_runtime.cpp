@@ -735,3 +735,294 @@ kf_status kf_jit_check(const kf_program* prog, const int32_t* plan, const kf_tar
 }
 
 }  // extern "C"
+
+// ============================================================================ a11: multi-GPU
+// Domain decomposition over a px x py process grid (x, y split; z whole; rank = iy*px + ix).
+// Each part runs the same plan on its local sub-domain; the periodic ghost fills of the
+// single-domain schedule become halo exchanges with the neighbouring parts (x strips first,
+// then y strips including the x ghosts, which covers corners).  Transports: loopback (all
+// parts in one process/GPU, strips copied device-to-device; used to test the decomposition
+// bit-exactly on one GPU) and NCCL send/recv (one process per GPU, NVLink/NVSwitch).
+#include <dlfcn.h>
+
+namespace kf {
+
+struct Nccl {
+  void* h = nullptr;
+  int (*getUniqueId)(void*) = nullptr;                          // ncclUniqueId* (128 bytes)
+  int (*commInitRank)(void**, int, const void*, int) = nullptr; // comm*, nranks, ncclUniqueId (by value: 128 B)
+  int (*send)(const void*, size_t, int, int, void*, cudaStream_t) = nullptr;
+  int (*recv)(void*, size_t, int, int, void*, cudaStream_t) = nullptr;
+  int (*groupStart)() = nullptr;
+  int (*groupEnd)() = nullptr;
+  int (*commDestroy)(void*) = nullptr;
+  const char* (*errStr)(int) = nullptr;
+};
+
+// ncclCommInitRank takes ncclUniqueId by value (struct of 128 chars): declare it that way.
+struct NcclId { char internal[128]; };
+
+static Nccl& nccl() {
+  static Nccl n;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_NOLOAD);   // prefer the copy already in the process
+    if (!h) h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) return;
+    n.h = h;
+    n.getUniqueId = (int (*)(void*))dlsym(h, "ncclGetUniqueId");
+    n.commInitRank = (int (*)(void**, int, const void*, int))dlsym(h, "ncclCommInitRank");
+    n.send = (int (*)(const void*, size_t, int, int, void*, cudaStream_t))dlsym(h, "ncclSend");
+    n.recv = (int (*)(void*, size_t, int, int, void*, cudaStream_t))dlsym(h, "ncclRecv");
+    n.groupStart = (int (*)())dlsym(h, "ncclGroupStart");
+    n.groupEnd = (int (*)())dlsym(h, "ncclGroupEnd");
+    n.commDestroy = (int (*)(void*))dlsym(h, "ncclCommDestroy");
+    n.errStr = (const char* (*)(int))dlsym(h, "ncclGetErrorString");
+  });
+  if (!n.h || !n.getUniqueId || !n.commInitRank || !n.send || !n.recv)
+    fail(KF_E_UNSUPPORTED, "NCCL (libnccl.so.2) not available");
+  return n;
+}
+
+static void ckn(int r, const char* what) {
+  if (r == 0) return;
+  fail(KF_E_NCCL, std::string(what) + ": " + (nccl().errStr ? nccl().errStr(r) : std::to_string(r)));
+}
+
+}  // namespace kf
+
+struct kf_dist {
+  std::vector<kf_exec*> parts;   // loopback: px*py parts; NCCL: 1 part
+  int px = 1, py = 1, rank = 0, world = 1;
+  bool use_nccl = false;
+  void* comm = nullptr;
+  void* stage = nullptr;         // NCCL staging (device): 4 strips of the largest face
+  uint64_t stage_bytes = 0;
+};
+
+namespace kf {
+
+static void dist_neighbors(int px, int py, int rank, int out[4]) {
+  const int ix = rank % px, iy = rank / px;
+  out[0] = iy * px + (ix + px - 1) % px;   // left  (x-)
+  out[1] = iy * px + (ix + 1) % px;        // right (x+)
+  out[2] = ((iy + py - 1) % py) * px + ix; // down  (y-)
+  out[3] = ((iy + 1) % py) * px + ix;      // up    (y+)
+}
+
+// Strip boxes of one buffer, in elements relative to the allocation base.
+struct Box { long long off; int w, h, d; };
+
+static void strip_boxes(const Program& p, int axis, Box* send_lo, Box* send_hi, Box* recv_lo, Box* recv_hi) {
+  const kf_layout& L = p.layout;
+  const int nx = int(p.n[0]), ny = int(p.n[1]), g0 = p.ghost[0], g1 = p.ghost[1];
+  const int d = int(p.n[2]) + 2 * p.ghost[2];
+  if (axis == 0) {
+    const int h = ny + 2 * g1;                    // every row, y ghosts included
+    const long long row0 = 0;
+    *send_lo = Box{row0 + L.xoff, g0, h, d};
+    *send_hi = Box{row0 + L.xoff + nx - g0, g0, h, d};
+    *recv_lo = Box{row0 + L.xoff - g0, g0, h, d};
+    *recv_hi = Box{row0 + L.xoff + nx, g0, h, d};
+  } else {
+    const int w = int(L.pitch);                   // whole padded rows: x ghosts (and corners) included
+    *send_lo = Box{(long long)g1 * L.pitch, w, g1, d};
+    *send_hi = Box{(long long)ny * L.pitch, w, g1, d};
+    *recv_lo = Box{0, w, g1, d};
+    *recv_hi = Box{(long long)(g1 + ny) * L.pitch, w, g1, d};
+  }
+}
+
+static void copy_box_buf(const Program& p, void* dst_base, const Box& db, const void* src_base, const Box& sb,
+                         cudaStream_t s) {
+  const kf_layout& L = p.layout;
+  CK(launch_copy_box((char*)dst_base + db.off * p.es, L.pitch, L.plane, (const char*)src_base + sb.off * p.es, L.pitch,
+                     L.plane, sb.w, sb.h, sb.d, p.es, s));
+}
+
+// Halo exchange of buffer id `b` on every part: decomposed axes exchange with neighbours,
+// other periodic axes wrap locally.
+static void dist_exchange(kf_dist* D, int b, cudaStream_t s) {
+  const Program& p = D->parts[0]->prog->p;
+  Geom gm = geom(p);
+  for (int axis = 0; axis < 3; axis++) {
+    if (p.bc[axis] != KF_BC_PERIODIC) continue;
+    const int np = axis == 0 ? D->px : (axis == 1 ? D->py : 1);
+    if (np == 1) {
+      for (kf_exec* E : D->parts) CK(launch_fill(axis, buf_ptr(E, b), p.es, gm, s));
+      continue;
+    }
+    Box slo, shi, rlo, rhi;
+    strip_boxes(p, axis, &slo, &shi, &rlo, &rhi);
+    if (!D->use_nccl) {
+      const int nparts = int(D->parts.size());
+      for (int r = 0; r < nparts; r++) {
+        int nb[4];
+        dist_neighbors(D->px, D->py, r, nb);
+        const int lo = axis == 0 ? nb[0] : nb[2], hi = axis == 0 ? nb[1] : nb[3];
+        // my low ghost <- low neighbour's high interior strip; my high ghost <- high neighbour's low strip
+        copy_box_buf(p, buf_ptr(D->parts[r], b), rlo, buf_ptr(D->parts[lo], b), shi, s);
+        copy_box_buf(p, buf_ptr(D->parts[r], b), rhi, buf_ptr(D->parts[hi], b), slo, s);
+      }
+    } else {
+      kf_exec* E = D->parts[0];
+      int nb[4];
+      dist_neighbors(D->px, D->py, D->rank, nb);
+      const int lo = axis == 0 ? nb[0] : nb[2], hi = axis == 0 ? nb[1] : nb[3];
+      const uint64_t strip = uint64_t(slo.w) * slo.h * slo.d * p.es;
+      char* st = (char*)D->stage;
+      char *s_lo = st, *s_hi = st + strip, *r_lo = st + 2 * strip, *r_hi = st + 3 * strip;
+      const kf_layout& L = p.layout;
+      auto pack = [&](char* dst, const Box& bx) {
+        CK(launch_copy_box(dst, bx.w, (long long)bx.w * bx.h, (const char*)buf_ptr(E, b) + bx.off * p.es, L.pitch, L.plane,
+                           bx.w, bx.h, bx.d, p.es, s));
+      };
+      auto unpack = [&](const Box& bx, const char* src) {
+        CK(launch_copy_box((char*)buf_ptr(E, b) + bx.off * p.es, L.pitch, L.plane, src, bx.w, (long long)bx.w * bx.h, bx.w,
+                           bx.h, bx.d, p.es, s));
+      };
+      pack(s_lo, slo);
+      pack(s_hi, shi);
+      Nccl& n = nccl();
+      ckn(n.groupStart(), "ncclGroupStart");
+      ckn(n.send(s_lo, strip, 1 /*ncclUint8*/, lo, D->comm, s), "ncclSend");   // my low strip -> low nbr's high ghost
+      ckn(n.send(s_hi, strip, 1, hi, D->comm, s), "ncclSend");                 // my high strip -> high nbr's low ghost
+      ckn(n.recv(r_hi, strip, 1, hi, D->comm, s), "ncclRecv");                 // high nbr's low strip -> my high ghost
+      ckn(n.recv(r_lo, strip, 1, lo, D->comm, s), "ncclRecv");                 // low nbr's high strip -> my low ghost
+      ckn(n.groupEnd(), "ncclGroupEnd");
+      unpack(rlo, r_lo);
+      unpack(rhi, r_hi);
+    }
+  }
+}
+
+static void dist_run(kf_dist* D, void* const* arrays, void* const* scratch, uint64_t scratch_bytes, int64_t nsteps,
+                     const double* params, cudaStream_t s) {
+  const Program& p = D->parts[0]->prog->p;
+  const int np = int(D->parts.size());
+  if (!arrays) fail(KF_E_ARG, "arrays is NULL");
+  for (int r = 0; r < np; r++) {
+    kf_exec* E = D->parts[r];
+    void* const* arr = arrays + size_t(r) * p.na;
+    for (int x = 0; x < p.na; x++)
+      if (!arr[x] || (reinterpret_cast<uintptr_t>(arr[x]) & 127)) fail(KF_E_ARG, "array pointers must be 128-byte aligned");
+    void* scr = scratch ? scratch[r] : nullptr;
+    if (scratch_bytes < E->scratch_bytes || (E->scratch_bytes && !scr))
+      fail(KF_E_RESOURCE, "scratch too small: need " + std::to_string(E->scratch_bytes) + " bytes per part");
+    ensure_device(E);
+    prepare_pointers(E, arr, scr, params);
+    std::vector<void*> av(arr, arr + p.na);
+    if (!E->scratch_vers.empty() && (E->shell_init_scratch != scr || E->shell_init_arrays != av)) {
+      Geom gm = geom(p);
+      for (size_t i = 0; i < E->scratch_vers.size(); i++)
+        CK(launch_copy_shell(buf_ptr(E, p.na + int(i)), arr[E->scratch_vers[i].x], p.es, gm, s));
+      E->shell_init_scratch = scr;
+      E->shell_init_arrays = av;
+    }
+  }
+  kf_exec* E0 = D->parts[0];
+  for (int b : E0->fill_all) dist_exchange(D, b, s);
+  for (int64_t step = 0; step < nsteps; step++) {
+    const int par = int(step % E0->period);
+    for (const Op& op : E0->sched[par]) {
+      if (op.kind == 0) dist_exchange(D, op.buf, s);
+      else
+        for (kf_exec* E : D->parts) launch_group(E, op.group, par, s);
+    }
+  }
+  if (E0->period == 2 && (nsteps % 2) == 1)
+    for (kf_exec* E : D->parts)
+      for (int x = 0; x < p.na; x++)
+        if (p.relaxed[x] && p.step_live[x]) {
+          int b = buffer_id(E, Ver{x, int(p.writers[x].size())}, 0);
+          CK(cudaMemcpyAsync(E->cur_arrays[x], buf_ptr(E, b), E->array_bytes, cudaMemcpyDeviceToDevice, s));
+        }
+  CK(cudaGetLastError());
+}
+
+}  // namespace kf
+
+extern "C" {
+
+kf_status kf_dist_unique_id(uint8_t id[128]) {
+  KF_TRY({
+    if (!id) fail(KF_E_ARG, "null argument");
+    NcclId u;
+    ckn(nccl().getUniqueId(&u), "ncclGetUniqueId");
+    std::memcpy(id, &u, 128);
+  });
+}
+
+kf_status kf_dist_neighbors(int32_t px, int32_t py, int32_t rank, int32_t out[4]) {
+  KF_TRY({
+    if (!out || px < 1 || py < 1 || rank < 0 || rank >= px * py) fail(KF_E_ARG, "bad process grid or rank");
+    int nb[4];
+    dist_neighbors(px, py, rank, nb);
+    for (int i = 0; i < 4; i++) out[i] = nb[i];
+  });
+}
+
+kf_status kf_dist_create(kf_exec* const* parts, int32_t n_parts, int32_t px, int32_t py, int32_t rank, int32_t world,
+                         const uint8_t* nccl_id, kf_dist** out) {
+  KF_TRY({
+    if (!parts || !out || n_parts < 1 || px < 1 || py < 1) fail(KF_E_ARG, "bad arguments");
+    auto D = std::make_unique<kf_dist>();
+    D->px = px;
+    D->py = py;
+    D->rank = rank;
+    D->world = world;
+    for (int i = 0; i < n_parts; i++) {
+      if (!parts[i]) fail(KF_E_ARG, "null part");
+      D->parts.push_back(parts[i]);
+    }
+    const Program& p = parts[0]->prog->p;
+    for (int i = 1; i < n_parts; i++)
+      if (parts[i]->prog != parts[0]->prog || parts[i]->plan.label != parts[0]->plan.label)
+        fail(KF_E_ARG, "all parts must run the same program and plan");
+    if ((px > 1 && p.bc[0] != KF_BC_PERIODIC) || (py > 1 && p.bc[1] != KF_BC_PERIODIC))
+      fail(KF_E_UNSUPPORTED, "decomposed axes must be PERIODIC in the local program (halo exchange replaces the wrap)");
+    if ((px > 1 && p.n[0] < p.ghost[0]) || (py > 1 && p.n[1] < p.ghost[1]))
+      fail(KF_E_ARG, "local extent smaller than the ghost width");
+    if (n_parts == px * py && world == 1) {
+      D->use_nccl = false;   // loopback: every part in this process
+    } else if (n_parts == 1 && world == px * py && rank >= 0 && rank < world) {
+      if (!nccl_id) fail(KF_E_ARG, "nccl_id required for the NCCL transport");
+      D->use_nccl = true;
+      NcclId u;
+      std::memcpy(&u, nccl_id, 128);
+      CK(cudaFree(nullptr));
+      // ncclCommInitRank(ncclComm_t*, int nranks, ncclUniqueId commId, int rank): id passed by value
+      auto init = (int (*)(void**, int, NcclId, int))nccl().commInitRank;
+      ckn(init(&D->comm, world, u, rank), "ncclCommInitRank");
+      const kf_layout& L = p.layout;
+      uint64_t fx = uint64_t(p.ghost[0]) * (p.n[1] + 2 * p.ghost[1]) * (p.n[2] + 2 * p.ghost[2]);
+      uint64_t fy = uint64_t(L.pitch) * p.ghost[1] * (p.n[2] + 2 * p.ghost[2]);
+      D->stage_bytes = 4 * std::max(fx, fy) * p.es;
+      if (cudaMalloc(&D->stage, D->stage_bytes) != cudaSuccess) fail(KF_E_OOM, "cudaMalloc (halo staging) failed");
+    } else {
+      fail(KF_E_ARG, "either n_parts == px*py with world == 1 (loopback) or n_parts == 1 with world == px*py (NCCL)");
+    }
+    *out = D.release();
+  });
+}
+
+kf_status kf_dist_run(kf_dist* d, void* const* arrays, void* const* scratch, uint64_t scratch_bytes, int64_t nsteps,
+                      const double* params, void* cuda_stream) {
+  KF_TRY({
+    if (!d) fail(KF_E_ARG, "null dist");
+    if (nsteps < 0) fail(KF_E_ARG, "nsteps < 0");
+    dist_run(d, arrays, scratch, scratch_bytes, nsteps, params, (cudaStream_t)cuda_stream);
+  });
+}
+
+void kf_dist_destroy(kf_dist* d) {
+  if (!d) return;
+  try {
+    if (d->comm && nccl().commDestroy) nccl().commDestroy(d->comm);
+    if (d->stage) cudaFree(d->stage);
+  } catch (...) {
+  }
+  delete d;
+}
+
+}  // extern "C"
