@@ -381,6 +381,16 @@ static void build_schedule(kf_exec* E) {
       }
       if (pass == 1) sched[par] = ops;
     }
+  // Buffers whose stored ghosts are read for in-group versions (frozen-boundary rule R9): their
+  // ghost cells on PERIODIC axes at frozen-ghost rows/planes are the wrap (or the neighbour's
+  // values in a decomposition) of never-written ghost rows, i.e. constant -- fill them once at
+  // the start of a run so kernels read them directly.
+  bool any_frozen = false, any_periodic = false;
+  for (int a = 0; a < 3; a++) (p.bc[a] == KF_BC_PERIODIC ? any_periodic : any_frozen) = true;
+  if (any_frozen && any_periodic)
+    for (int par = 0; par < E->period; par++)
+      for (const GroupExec& g : E->G)
+        for (const Ver& v : g.mids) all_fill.insert(buffer_id(E, v, par));
   E->sched = sched;
   E->fill_all.assign(all_fill.begin(), all_fill.end());
 }
