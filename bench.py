@@ -62,9 +62,10 @@ def choose_plan(prog, target, which: str):
     if which == "hand":
         from workloads.programs import weather_hand_plan
         return weather_hand_plan(prog.desc), "hand plan (App. A.4)"
-    method = kf.SEARCH_BRUTE if n <= 10 else kf.SEARCH_GREEDY
+    method = kf.SEARCH_BRUTE_TIME if n <= 10 else kf.SEARCH_GREEDY_TIME
     plan, _ = prog.search(method, target)
-    return plan, ("brute-force optimum" if method == kf.SEARCH_BRUTE else "greedy search")
+    return plan, ("brute-force on projected time" if method == kf.SEARCH_BRUTE_TIME
+                  else "greedy search on the resource-aware projected time")
 
 
 # ---------------------------------------------------------------- clocks
@@ -173,31 +174,6 @@ def cpu_baseline(name: str, budget_s: float = 12.0):
 
 
 # ---------------------------------------------------------------- GPU timing
-def time_plan(ex, dev, scratch, steps, warmup, stream, profile=False):
-    import torch
-    if profile:
-        ex.set_profiling(True)
-    ex.run(dev, scratch, warmup, stream=stream)
-    torch.cuda.synchronize()
-    if profile:
-        ex.set_profiling(True)    # reset accumulators after warm-up
-    if torch.distributed.is_initialized():
-        torch.distributed.barrier()
-    torch.cuda.synchronize()
-    e0 = torch.cuda.Event(enable_timing=True)
-    e1 = torch.cuda.Event(enable_timing=True)
-    e0.record(stream)
-    ex.run(dev, scratch, steps, stream=stream)
-    e1.record(stream)
-    torch.cuda.synchronize()
-    ms = e0.elapsed_time(e1)
-    gt = None
-    if profile:
-        gt = ex.group_times()
-        ex.set_profiling(False)
-    return ms, gt
-
-
 AUTOTUNE_CANDIDATES = [((64, 4, 0), 2, 1), ((64, 4, 0), 2, 2), ((32, 8, 0), 2, 1), ((32, 8, 0), 2, 2),
                        ((64, 4, 0), 3, 1), ((32, 8, 0), 3, 1), ((32, 4, 0), 2, 1), ((64, 8, 0), 2, 1)]
 
@@ -244,20 +220,71 @@ def max_over_ranks(x: float) -> float:
     return x
 
 
+class Runner:
+    """One rank's view of the hot path: a kf.Exec (1 GPU) or a kf.Dist over NCCL (N GPUs)."""
+
+    def __init__(self, prog, plan, target, group_targets, dist_info):
+        import torch
+        import paper_conf_sc_wahibm14_b200 as kf
+        self.ex = kf.Exec(prog, plan, target, group_targets=group_targets)
+        sb = self.ex.scratch_bytes()
+        self.scratch = torch.empty(sb, dtype=torch.uint8, device="cuda") if sb else None
+        self.dist = None
+        if dist_info is not None:
+            px, py, rank, world, nid = dist_info
+            self.dist = kf.Dist([self.ex], px, py, rank, world, nid)
+
+    def run(self, dev, nsteps, stream):
+        if self.dist is None:
+            self.ex.run(dev, self.scratch, nsteps, stream=stream)
+        else:
+            self.dist.run([dev], [self.scratch], nsteps, stream=stream)
+
+
+def time_runner(rn, dev, steps, warmup, stream, profile=False):
+    import torch
+    rn.run(dev, warmup, stream)
+    torch.cuda.synchronize()
+    if profile:
+        rn.ex.set_profiling(True)
+    if torch.distributed.is_initialized():
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    rn.run(dev, steps, stream)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1)
+    gt = None
+    if profile:
+        gt = rn.ex.group_times()
+        rn.ex.set_profiling(False)
+    return ms, gt
+
+
+def grid_for(world):
+    return {1: (1, 1), 2: (2, 1), 4: (2, 2), 8: (4, 2)}.get(world, (world, 1))
+
+
 def run_kf(args):
     import numpy as np
     import torch
     import paper_conf_sc_wahibm14_b200 as kf
+    from workloads.program import PROG_RELAX_ALL
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if world > 1:
         torch.cuda.set_device(local)
-        torch.distributed.init_process_group("nccl")
+        torch.distributed.init_process_group("nccl", device_id=torch.device("cuda", local))
     else:
         torch.cuda.set_device(0)
     desc, gen, tkw, label = workload(args.workload)
+    if args.relax_all and desc.name == "weather":
+        desc = desc.with_(flags=PROG_RELAX_ALL)
     if args.tile:
         tkw["tile"] = tuple(int(v) for v in args.tile.split(","))
     if args.stages:
@@ -265,58 +292,84 @@ def run_kf(args):
     if args.threads:
         tkw["threads"] = args.threads
     target = kf.Target(**tkw)
-    prog = kf.Program(desc)
+    prog = kf.Program(desc)          # the per-GPU sub-domain program (weak scaling)
     plan, plan_kind = choose_plan(prog, target, args.plan)
+    dist_info = None
+    if world > 1:
+        px, py = grid_for(world)
+        nid = kf.dist_unique_id() if rank == 0 else bytes(128)
+        t = torch.tensor(list(nid), dtype=torch.uint8, device="cuda")
+        torch.distributed.broadcast(t, 0)
+        dist_info = (px, py, rank, world, bytes(t.cpu().tolist()))
     # synthetic inputs of the paper-shaped workload (seed 3 + rank: each rank owns its sub-domain)
     inputs = gen(desc, 3 + rank)
     dev = kf.device_arrays(prog, inputs)
     del inputs
-    t0 = time.time()
-    tuned = None
-    if args.autotune:
-        gtargets, tuned, _ = autotune(prog, plan, dev, tkw)
-        ex = kf.Exec(prog, plan, target, group_targets=gtargets)
-    else:
-        ex = kf.Exec(prog, plan, target)
-    jit_s = time.time() - t0
-    sb = ex.scratch_bytes()
-    scratch = torch.empty(sb, dtype=torch.uint8, device="cuda") if sb else None
     stream = torch.cuda.current_stream()
-    info = ex.info()
+    t0 = time.time()
+    tuned, gtargets = None, None
+    if args.autotune:
+        if rank == 0:
+            gtargets, tuned, _ = autotune(prog, plan, dev, tkw)
+        if world > 1:
+            obj = [tuned]
+            torch.distributed.broadcast_object_list(obj, 0)
+            tuned = obj[0]
+            gtargets = [kf.Target(**dict(tkw, tile=tuple(c[0]), stages=c[1], zunroll=c[2])) for c in tuned]
+    rn = Runner(prog, plan, target, gtargets, dist_info)
+    jit_s = time.time() - t0
+    info = rn.ex.info()
     npts = desc.npts
 
     with ClockSampler(local) as clk:
-        ms, _ = time_plan(ex, dev, scratch, args.steps, args.warmup, stream)
+        ms, _ = time_runner(rn, dev, args.steps, args.warmup, stream)
     ms = max_over_ranks(ms)
     clocks = clk.summary()
     # per-group device times over a second timed region (events on the launch stream)
-    ms_prof, (gms, nlaunch) = time_plan(ex, dev, scratch, args.steps, max(1, args.warmup // 2), stream, profile=True)
+    ms_prof, (gms, nlaunch) = time_runner(rn, dev, args.steps, 1, stream, profile=True)
     # unfused plan on the same inputs: speedup vs unfused
     unf = None
     if not args.no_unfused and args.plan != "unfused":
-        ex_u = kf.Exec(prog, list(range(prog.nk)), target)
-        sb_u = ex_u.scratch_bytes()
-        scr_u = torch.empty(sb_u, dtype=torch.uint8, device="cuda") if sb_u else None
-        ms_u, _ = time_plan(ex_u, dev, scr_u, args.steps, args.warmup, stream)
+        rn_u = Runner(prog, list(range(prog.nk)), target, None, dist_info)
+        ms_u, _ = time_runner(rn_u, dev, args.steps, args.warmup, stream)
         ms_u = max_over_ranks(ms_u)
-        unf = {"ms_per_step": ms_u / args.steps, "bytes_per_step": ex_u.info().compulsory_bytes_per_step}
-        del ex_u, scr_u
-    # end-to-end through the C ABI with host buffers (copies inside the timed region)
+        unf = {"ms_per_step": ms_u / args.steps, "bytes_per_step": rn_u.ex.info().compulsory_bytes_per_step}
+        del rn_u
+    # end-to-end through the public API with host buffers (copies inside the timed region)
     e2e = None
     if not args.no_e2e:
-        host = [t.cpu().pin_memory() for t in dev]
-        ex.run_host([h.data_ptr() for h in host], 1, stream=stream.cuda_stream)   # warm (allocs, first full upload)
-        torch.cuda.synchronize()
         k = max(1, min(args.steps, 3))
-        t0 = time.perf_counter()
-        h2d = d2h = 0
-        for _ in range(k):
-            a, b = ex.run_host([h.data_ptr() for h in host], 1, stream=stream.cuda_stream)
-            h2d, d2h = a, b
-        dt = time.perf_counter() - t0
+        if rn.dist is None:
+            host = [t.cpu().pin_memory() for t in dev]
+            rn.ex.run_host([h.data_ptr() for h in host], 1, stream=stream.cuda_stream)   # warm (allocs, full upload)
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            h2d = d2h = 0
+            for _ in range(k):
+                h2d, d2h = rn.ex.run_host([h.data_ptr() for h in host], 1, stream=stream.cuda_stream)
+            dt = time.perf_counter() - t0
+            how = "kf_run_host (C ABI, pinned host buffers), host wall clock, synchronising"
+        else:
+            ins = [x for x in range(len(desc.arrays)) if prog.array_info(x).upward_exposed]
+            outs = [x for x in range(len(desc.arrays)) if prog.array_info(x).step_live]
+            host = {x: dev[x].cpu().pin_memory() for x in set(ins) | set(outs)}
+            torch.cuda.synchronize()
+            torch.distributed.barrier()
+            t0 = time.perf_counter()
+            for _ in range(k):
+                for x in ins:
+                    dev[x].copy_(host[x], non_blocking=True)
+                rn.run(dev, 1, stream)
+                for x in outs:
+                    host[x].copy_(dev[x], non_blocking=True)
+                torch.cuda.synchronize()
+            dt = time.perf_counter() - t0
+            h2d = sum(host[x].numel() * host[x].element_size() for x in ins)
+            d2h = sum(host[x].numel() * host[x].element_size() for x in outs)
+            how = "kf.Dist.run with pinned host buffers copied in/out every step, host wall clock"
         dt = max_over_ranks(dt)
         e2e = {"value": world * npts * k / dt, "unit": UNIT, "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
-               "steps": k, "timing": "host wall clock around kf_run_host (synchronising), max over ranks"}
+               "steps": k, "timing": how + ", max over ranks"}
         del host
 
     bytes_step = info.compulsory_bytes_per_step
@@ -324,11 +377,9 @@ def run_kf(args):
     peaks = measured_peaks()
     hbm_peak = peaks["hbm_gbs"] if peaks and "hbm_gbs" in peaks else 6650.0
     peak_src = "MEASURED_PEAKS.json hbm_gbs" if peaks else "B200_PROFILING.md fallback 6.65 TB/s"
-    # dominant kernel = the group with the largest device time
     g_dom = int(np.argmax(gms))
-    gi = ex.group_info(g_dom)
+    gi = rn.ex.group_info(g_dom)
     gname = gi.name.decode() if isinstance(gi.name, bytes) else gi.name
-    launches_dom = args.steps * info.period // info.period
     t_launch_ms = gms[g_dom] / args.steps
     achieved = gi.bytes_per_launch / (t_launch_ms / 1e3) / 1e9
     roofline = {"bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s", "frac": achieved / hbm_peak,
@@ -337,22 +388,25 @@ def run_kf(args):
                 "algorithmic_bytes_per_launch": gi.bytes_per_launch,
                 "per_group_ms_per_step": [g / args.steps for g in gms]}
     achieved_step = bytes_step / (ms / args.steps / 1e3) / 1e9
-    _, _, t_proj = prog.project(plan, target)
+    per, _, t_proj = prog.project(plan, target)
     res = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
         "dtype": "f64" if desc.dtype == 1 else "f32", "data": "synthetic (seeded, paper-shaped fields)",
-        "config": {"workload": label, "plan": f"{plan_kind}: {info.n_groups} fused groups of {prog.nk} kernels",
+        "config": {"workload": label + (" with RELAX_ALL renaming" if desc.flags & 2 else ""),
+                   "plan": f"{plan_kind}: {info.n_groups} fused groups of {prog.nk} kernels",
                    "plan_labels": plan, "tile": list(target.tile), "stages": target.stages,
                    "threads": target.threads, "l2": "inputs larger than L2 (each array > 126 MB), no flush",
-                   "parallelism": f"replicas x{world}" if world > 1 else "1 GPU",
-                   "graph": True, "jit_s": round(jit_s, 2),
+                   "parallelism": (f"xy domain decomposition {grid_for(world)[0]}x{grid_for(world)[1]}, NCCL halo "
+                                   f"exchange, weak (512x512x128 per GPU)") if world > 1 else "1 GPU",
+                   "graph": world == 1, "jit_s": round(jit_s, 2),
                    "per_group_launch_config": tuned if tuned else "uniform"},
         "hbm_gbs_compulsory": achieved_step,
         "frac_of_measured_copy": achieved_step / hbm_peak,
         "frac_of_nominal_8TBs": achieved_step / 8000.0,
         "compulsory_bytes_per_step": bytes_step,
         "projected_ms_per_step": t_proj * 1e3,
+        "model_ms_per_step": sum(g.t_model_s for g in per) * 1e3,
         "roofline": roofline,
         "gpu_launches": int(info.launches_per_step * args.steps),
         "clocks": clocks,
@@ -420,7 +474,8 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="kf", choices=["kf", "reference"])
     ap.add_argument("--workload", default="weather")
-    ap.add_argument("--plan", default="hand", choices=["best", "unfused", "hand"])
+    ap.add_argument("--plan", default="best", choices=["best", "unfused", "hand"])
+    ap.add_argument("--relax-all", type=int, default=1, help="weather: rename every written array (KF_PROG_RELAX_ALL)")
     ap.add_argument("--tile", default=None)
     ap.add_argument("--stages", type=int, default=None)
     ap.add_argument("--threads", type=int, default=None)

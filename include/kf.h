@@ -133,9 +133,10 @@ kf_status kf_program_edges(const kf_program* prog, kf_edge* out, int32_t cap, in
 kf_status kf_program_reach(const kf_program* prog, uint8_t* reach);
 
 /* Array classes: RO never written; WO written never read; EXPANDABLE >= 2
- * writing kernels; RW otherwise.  Also: renamed (relaxed) flag and step-live flag (R15). */
+ * writing kernels; RW otherwise.  Also: renamed (relaxed) flag, step-live flag (R15) and
+ * upward_exposed (read before any write in a step = an input of every step). */
 typedef enum { KF_CLS_RO = 0, KF_CLS_RW = 1, KF_CLS_EXPANDABLE = 2, KF_CLS_WO = 3 } kf_array_class;
-typedef struct { int32_t cls, n_writers, n_readers, relaxed, step_live, pad; } kf_array_info;
+typedef struct { int32_t cls, n_writers, n_readers, relaxed, step_live, upward_exposed; } kf_array_info;
 kf_status kf_program_array_info(const kf_program* prog, int32_t array, kf_array_info* out);
 
 /* Degree of kinship (Table II) of kernels a and b inside `group` (R5: the chain

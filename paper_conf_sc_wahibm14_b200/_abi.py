@@ -52,7 +52,7 @@ class kf_edge(C.Structure):
 
 class kf_array_info(C.Structure):
     _fields_ = [("cls", C.c_int32), ("n_writers", C.c_int32), ("n_readers", C.c_int32), ("relaxed", C.c_int32),
-                ("step_live", C.c_int32), ("pad", C.c_int32)]
+                ("step_live", C.c_int32), ("upward_exposed", C.c_int32)]
 
 
 class kf_layout(C.Structure):

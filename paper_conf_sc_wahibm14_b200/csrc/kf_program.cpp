@@ -292,6 +292,7 @@ kf_status kf_program_array_info(const kf_program* prog, int32_t x, kf_array_info
     r.n_readers = int(p.readers[x].size());
     r.relaxed = p.relaxed[x];
     r.step_live = p.step_live[x];
+    r.upward_exposed = p.readers_of_version(x, 0).empty() ? 0 : 1;
     *out = r;
   });
 }

@@ -935,9 +935,29 @@ static void dist_run(kf_dist* D, void* const* arrays, void* const* scratch, uint
   for (int64_t step = 0; step < nsteps; step++) {
     const int par = int(step % E0->period);
     for (const Op& op : E0->sched[par]) {
-      if (op.kind == 0) dist_exchange(D, op.buf, s);
-      else
-        for (kf_exec* E : D->parts) launch_group(E, op.group, par, s);
+      if (op.kind == 0) {
+        dist_exchange(D, op.buf, s);
+      } else {
+        for (kf_exec* E : D->parts) {
+          if (!E->profiling) {
+            launch_group(E, op.group, par, s);
+            continue;
+          }
+          cudaEvent_t a, b;
+          if (E->evpool.size() >= 2) {
+            a = E->evpool.back(); E->evpool.pop_back();
+            b = E->evpool.back(); E->evpool.pop_back();
+          } else {
+            CK(cudaEventCreate(&a));
+            CK(cudaEventCreate(&b));
+          }
+          CK(cudaEventRecord(a, s));
+          launch_group(E, op.group, par, s);
+          CK(cudaEventRecord(b, s));
+          E->pending.emplace_back(op.group, a, b);
+          E->launches++;
+        }
+      }
     }
   }
   if (E0->period == 2 && (nsteps % 2) == 1)

@@ -144,8 +144,8 @@ def test_per_group_launch_configs():
     ref = interp.run(desc, inputs, 2)
     plan = weather_hand_plan(desc)
     m = max(plan) + 1
-    cfgs = [((64, 4, 0), 2, 1, (1, 1), 256), ((32, 8, 0), 2, 2, (2, 1), 128), ((16, 8, 3), 3, 1, (1, 2), 64),
-            ((32, 4, 0), 2, 3, (2, 1), 64), ((64, 8, 0), 2, 1, (2, 2), 128)]
+    cfgs = [((64, 4, 0), 2, 1, (1, 1), 256), ((32, 8, 0), 2, 2, (2, 1), 256), ((16, 8, 3), 3, 1, (1, 2), 64),
+            ((32, 4, 0), 2, 3, (1, 1), 128), ((64, 8, 0), 2, 1, (2, 2), 256)]
     tg = [kf.Target(tile=cfgs[g % 5][0], stages=cfgs[g % 5][1], zunroll=cfgs[g % 5][2], pblock=cfgs[g % 5][3],
                     threads=cfgs[g % 5][4]) for g in range(m)]
     prog = kf.Program(desc)
