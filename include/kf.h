@@ -226,7 +226,9 @@ typedef enum {
   KF_SEARCH_GREEDY = 1,  /* agglomerative merging of groups by largest byte saving          */
   KF_SEARCH_AUTO = 2,    /* brute if n <= 10 else greedy                                    */
   KF_SEARCH_GREEDY_TIME = 3,  /* greedy merging on the resource-aware projected time (R22)    */
-  KF_SEARCH_BRUTE_TIME = 4    /* brute force on the resource-aware projected time (n <= 14)    */
+  KF_SEARCH_BRUTE_TIME = 4,   /* brute force on the resource-aware projected time (n <= 14)    */
+  KF_SEARCH_HGGA = 5,         /* hybrid grouping GA (Alg. 1) on projected time; seed  */
+  KF_SEARCH_HGGA_BYTES = 6    /* the same GA on compulsory bytes (comparable to BRUTE)           */
 } kf_search_method;
 /* Minimises total compulsory bytes (or, for the *_TIME methods, total projected time) over
  * legal plans; ties -> lexicographically smallest canonical labels (R17).  plan_out:

@@ -12,7 +12,7 @@ from ._abi import (check, kf_access, kf_array_desc, kf_array_info, kf_edge, kf_e
                    kf_group_proj, kf_insn, kf_kernel_desc, kf_kernel_sched, kf_layout, kf_program_desc,
                    kf_program_info, kf_stmt, kf_target, kf_violation, lib)
 
-SEARCH_BRUTE, SEARCH_GREEDY, SEARCH_AUTO, SEARCH_GREEDY_TIME, SEARCH_BRUTE_TIME = 0, 1, 2, 3, 4
+SEARCH_BRUTE, SEARCH_GREEDY, SEARCH_AUTO, SEARCH_GREEDY_TIME, SEARCH_BRUTE_TIME, SEARCH_HGGA, SEARCH_HGGA_BYTES = range(7)
 
 
 def _i32(seq) -> C.Array:

@@ -11,6 +11,7 @@
 // ties -> lexicographically smallest canonical labels (R17).
 #include <algorithm>
 #include <functional>
+#include <random>
 #include <unordered_map>
 
 #include "kf_internal.hpp"
@@ -184,6 +185,204 @@ static std::vector<int> greedy(const Program& p, Evaluator& ev, uint64_t* best_b
   return label;
 }
 
+// ---------------------------------------------------------------- HGGA (NEXT-1)
+// Hybrid Grouping Genetic Algorithm (Alg. 1; Falkenauer [19]): individuals
+// are partitions whose genes are the groups (new kernels).  Group-aware crossover injects a
+// random subset of the other parent's groups and repairs the rest; mutation dissolves or merges
+// groups; every offspring is made legal (infeasible groups fall back to singletons, the first
+// violated constraint rejects a merge -- the paper's active-constraint pruning) and then
+// locally improved by legal merges.  Deterministic for a given seed.
+struct Indiv {
+  std::vector<int> lab;
+  double cost = 0;
+};
+
+class Hgga {
+ public:
+  Hgga(const Program& p, Evaluator& ev, bool by_time, uint64_t seed) : p_(p), ev_(ev), by_time_(by_time), rng_(seed) {}
+
+  std::vector<int> run(int pop_size, int max_gen, int stall_gen, uint64_t* bytes_out) {
+    std::vector<Indiv> pop;
+    for (int i = 0; i < pop_size; i++) pop.push_back(random_individual(i == 0 ? 0.0 : 0.6));
+    auto better = [](const Indiv& a, const Indiv& b) { return a.cost < b.cost || (a.cost == b.cost && a.lab < b.lab); };
+    Indiv best = *std::min_element(pop.begin(), pop.end(), better);
+    int stall = 0;
+    for (int gen = 0; gen < max_gen && stall < stall_gen; gen++) {
+      std::vector<Indiv> next;
+      // elitism: keep the two best
+      std::sort(pop.begin(), pop.end(), better);
+      next.push_back(pop[0]);
+      if (pop.size() > 1) next.push_back(pop[1]);
+      while (int(next.size()) < pop_size) {
+        const Indiv& a = tournament(pop);
+        const Indiv& b = tournament(pop);
+        Indiv c = crossover(a, b);
+        if (uni() < 0.3) c = mutate(c);
+        next.push_back(c);
+      }
+      pop = std::move(next);
+      Indiv gb = *std::min_element(pop.begin(), pop.end(), better);
+      if (better(gb, best)) {
+        best = gb;
+        stall = 0;
+      } else {
+        stall++;
+      }
+    }
+    if (bytes_out) {
+      uint64_t b = 0;
+      ev_.legal(best.lab, nm(best.lab), &b);
+      *bytes_out = b;
+    }
+    return best.lab;
+  }
+
+ private:
+  const Program& p_;
+  Evaluator& ev_;
+  bool by_time_;
+  std::mt19937_64 rng_;
+
+  double uni() { return std::uniform_real_distribution<double>(0.0, 1.0)(rng_); }
+  int rint(int n) { return int(std::uniform_int_distribution<int>(0, n - 1)(rng_)); }
+  static int nm(const std::vector<int>& lab) { return *std::max_element(lab.begin(), lab.end()) + 1; }
+
+  bool cost(const std::vector<int>& lab, double* c) {
+    uint64_t b = 0;
+    double t = 0;
+    if (!ev_.legal(lab, nm(lab), &b, &t)) return false;
+    *c = by_time_ ? t : double(b);
+    return true;
+  }
+  std::vector<std::vector<int>> groups(const std::vector<int>& lab) {
+    std::vector<std::vector<int>> gs(nm(lab));
+    for (int k = 0; k < p_.nk; k++) gs[lab[k]].push_back(k);
+    return gs;
+  }
+  static std::vector<int> from_groups(const std::vector<std::vector<int>>& gs, int n) {
+    std::vector<int> lab(n, -1);
+    int g = 0;
+    for (auto& grp : gs)
+      if (!grp.empty()) {
+        for (int k : grp) lab[k] = g;
+        g++;
+      }
+    return canon(lab, nullptr);
+  }
+  // Make a plan legal: groups that are illegal alone dissolve into singletons; a cyclic quotient
+  // dissolves groups until acyclic.
+  std::vector<int> repair(std::vector<std::vector<int>> gs) {
+    std::vector<std::vector<int>> out;
+    for (auto& g : gs) {
+      if (g.empty()) continue;
+      std::sort(g.begin(), g.end());
+      if (g.size() == 1 || ev_.eval(g).ok) out.push_back(g);
+      else
+        for (int k : g) out.push_back({k});
+    }
+    std::vector<int> lab = from_groups(out, p_.nk);
+    while (!quotient_acyclic(p_, lab, nm(lab), nullptr)) {
+      int bad = -1;
+      quotient_acyclic(p_, lab, nm(lab), &bad);
+      auto g2 = groups(lab);
+      std::vector<std::vector<int>> o2;
+      for (int i = 0; i < int(g2.size()); i++) {
+        if (i == bad)
+          for (int k : g2[i]) o2.push_back({k});
+        else
+          o2.push_back(g2[i]);
+      }
+      lab = from_groups(o2, p_.nk);
+    }
+    return lab;
+  }
+  // Local improvement: randomized legal merges of adjacent groups that lower the cost.
+  Indiv improve(std::vector<int> lab, int tries) {
+    double c = 0;
+    cost(lab, &c);
+    for (int t = 0; t < tries; t++) {
+      auto gs = groups(lab);
+      if (gs.size() < 2) break;
+      int gi = rint(int(gs.size()));
+      std::vector<int> cand;
+      for (int gj = 0; gj < int(gs.size()); gj++) {
+        if (gj == gi) continue;
+        bool adj = false;
+        for (int a : gs[gi]) {
+          for (int b : gs[gj])
+            if (p_.share[a][b]) { adj = true; break; }
+          if (adj) break;
+        }
+        if (adj) cand.push_back(gj);
+      }
+      if (cand.empty()) continue;
+      int gj = cand[rint(int(cand.size()))];
+      std::vector<int> l2 = lab;
+      for (int k = 0; k < p_.nk; k++)
+        if (l2[k] == gj) l2[k] = gi;
+      l2 = canon(l2, nullptr);
+      double c2;
+      if (cost(l2, &c2) && c2 < c) { lab = l2; c = c2; }
+    }
+    return Indiv{lab, c};
+  }
+  Indiv random_individual(double merge_p) {
+    std::vector<int> lab(p_.nk);
+    for (int k = 0; k < p_.nk; k++) lab[k] = k;
+    if (merge_p > 0) {
+      // random legal merges (not necessarily improving): diversity of the initial population
+      for (int t = 0; t < 3 * p_.nk; t++) {
+        if (uni() > merge_p) continue;
+        int a = rint(p_.nk), b = rint(p_.nk);
+        if (lab[a] == lab[b] || !p_.share[a][b]) continue;
+        std::vector<int> l2 = lab;
+        int ga = lab[a], gb = lab[b];
+        for (int k = 0; k < p_.nk; k++)
+          if (l2[k] == gb) l2[k] = ga;
+        l2 = canon(l2, nullptr);
+        double c2;
+        if (cost(l2, &c2)) lab = l2;
+      }
+    }
+    return improve(canon(lab, nullptr), p_.nk);
+  }
+  const Indiv& tournament(const std::vector<Indiv>& pop) {
+    const Indiv& a = pop[rint(int(pop.size()))];
+    const Indiv& b = pop[rint(int(pop.size()))];
+    return (a.cost < b.cost || (a.cost == b.cost && a.lab < b.lab)) ? a : b;
+  }
+  Indiv crossover(const Indiv& A, const Indiv& B) {
+    auto ga = groups(A.lab), gb = groups(B.lab);
+    // inject a random subset of B's multi-kernel groups
+    std::vector<std::vector<int>> inj;
+    for (auto& g : gb)
+      if (g.size() > 1 && uni() < 0.5) inj.push_back(g);
+    std::vector<char> taken(p_.nk, 0);
+    for (auto& g : inj)
+      for (int k : g) taken[k] = 1;
+    std::vector<std::vector<int>> out = inj;
+    for (auto& g : ga) {
+      std::vector<int> rest;
+      for (int k : g)
+        if (!taken[k]) rest.push_back(k);
+      if (!rest.empty()) out.push_back(rest);
+    }
+    return improve(repair(out), p_.nk / 2 + 1);
+  }
+  Indiv mutate(const Indiv& A) {
+    auto gs = groups(A.lab);
+    std::vector<std::vector<int>> out;
+    int victim = rint(int(gs.size()));
+    for (int i = 0; i < int(gs.size()); i++) {
+      if (i == victim && gs[i].size() > 1)
+        for (int k : gs[i]) out.push_back({k});   // dissolve a group
+      else
+        out.push_back(gs[i]);
+    }
+    return improve(repair(out), p_.nk / 2 + 1);
+  }
+};
+
 }  // namespace kf
 
 using namespace kf;
@@ -220,6 +419,10 @@ kf_status kf_plan_search(const kf_program* prog, const kf_target* target, int32_
       if (!ev.legal(best, *std::max_element(best.begin(), best.end()) + 1, nullptr))
         fail(KF_E_ILLEGAL_PLAN, "even the unfused plan is illegal under this target");
       (void)m;
+    } else if (method == KF_SEARCH_HGGA || method == KF_SEARCH_HGGA_BYTES) {
+      // population 100 as in Table VI; stop after 30 generations without improvement
+      Hgga h(p, ev, method == KF_SEARCH_HGGA, seed);
+      best = h.run(100, 2000, 30, &best_b);
     } else {
       fail(KF_E_ARG, "unknown search method");
     }

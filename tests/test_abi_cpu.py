@@ -153,3 +153,58 @@ def test_codegen_compiles_for_sm100a():
             assert "sm_100a" in log
             assert spill == 0
             assert 0 < regs <= per[g].regs_est, (regs, per[g].regs_est)
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_suite_generator_programs_match_oracle(seed):
+    """Config 2 generator (App. A.3, Table V shape) at 7 kernels: legality of every partition,
+    bytes and the optimum match the oracle's brute force."""
+    desc = P.gen_suite(n_kernels=7, n_arrays=6, seed=seed, n=(16, 16, 8))
+    p = kf.Program(desc)
+    legal_o = En.legal_plans(desc)
+    assert p.count_legal() == len(legal_o)
+    plan, b = p.search(kf.SEARCH_BRUTE)
+    bo, bb = En.best_plan(desc)
+    assert plan == bo and b == bb
+
+
+def test_suite_generator_config2_shape():
+    """10 kernels / 8 arrays, mixed 7/13/27-point stencils, every shared array in 2..8 kernels."""
+    for seed in range(4):
+        desc = P.gen_suite(seed=seed)
+        assert len(desc.kernels) == 10 and len(desc.arrays) == 8
+        p = kf.Program(desc)
+        n = p.count_legal()
+        assert 1 <= n <= 5000
+        plan, b = p.search(kf.SEARCH_BRUTE)
+        assert b < p.project(list(range(10)))[1]
+
+
+def test_hgga_finds_brute_force_optimum_and_is_deterministic():
+    """NEXT-1: the HGGA (Alg. 1) verified by the deterministic method on small
+    benchmarks; repeated seeded runs return the same plan."""
+    for seed in range(4):
+        desc = P.gen_suite(seed=seed)
+        p = kf.Program(desc)
+        _, b_opt = p.search(kf.SEARCH_BRUTE)
+        plans = [p.search(kf.SEARCH_HGGA_BYTES, seed=7) for _ in range(3)]
+        assert all(pl == plans[0] for pl in plans)
+        assert plans[0][1] == b_opt
+        assert p.validate(plans[0][0])[0] == 0
+    hits = 0
+    for seed in range(6):
+        desc = P.random_program(50 + seed, nk=7, na=4)
+        p = kf.Program(desc)
+        hits += p.search(kf.SEARCH_HGGA_BYTES, seed=1)[1] == p.search(kf.SEARCH_BRUTE)[1]
+    assert hits >= 5
+
+
+def test_hgga_weather_no_worse_than_greedy():
+    desc = P.weather(n=(64, 64, 32))
+    p = kf.Program(desc)
+    plan_h, _ = p.search(kf.SEARCH_HGGA, seed=3)
+    plan_g, _ = p.search(kf.SEARCH_GREEDY_TIME)
+    assert p.validate(plan_h)[0] == 0
+    th = sum(g.t_model_s for g in p.project(plan_h)[0])
+    tg = sum(g.t_model_s for g in p.project(plan_g)[0])
+    assert th <= tg * 1.0001

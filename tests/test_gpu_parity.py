@@ -156,3 +156,44 @@ def test_per_group_launch_configs():
     ex.run(dev, scratch, 2)
     torch.cuda.synchronize()
     assert compare(desc, kf.host_arrays(prog, dev), ref) == []
+
+
+def test_suite_config2_every_legal_plan():
+    """BASELINE config 2 shape (10 kernels / 8 arrays, mixed 7/13/27-point fp32 stencils, periodic
+    xy): every legal plan of a generated program runs bit-exactly (grid reduced to 40x32x12)."""
+    desc = P.gen_suite(seed=1, n=(40, 32, 12))
+    inputs = D.uniform(desc, 2)
+    ref = interp.run(desc, inputs, 3)
+    prog = kf.Program(desc)
+    legal = En.legal_plans(desc) if False else None
+    n = prog.count_legal()
+    assert n == 188
+    # enumerate through the oracle's restricted-growth strings, keeping the library-legal ones
+    tgt = kf.Target(tile=(16, 8, 0))
+    checked = 0
+    for plan in En.restricted_growth(10):
+        if prog.validate(plan, tgt)[0] != 0:
+            continue
+        got, _ = run_kf(desc, plan, inputs, 3, tgt)
+        assert compare(desc, got, ref) == [], plan
+        checked += 1
+    assert checked == prog.count_legal(tgt)
+
+
+@pytest.mark.parametrize("tile", [(32, 8, 0), (16, 8, 0)])
+def test_stress_config5_radius4_plans(tile):
+    """BASELINE config 5 shape: radius-4 (25-point) fp64 stencils L25(L25(f)) + update, RELAX_ALL,
+    ghost 8, periodic xy; every legal plan (the fully fused group sits near the SMEM limit)."""
+    desc = P.stress(m=2, n=(40, 36, 20))
+    inputs = D.uniform(desc, 5)
+    ref = interp.run(desc, inputs, 2)
+    prog = kf.Program(desc)
+    tgt = kf.Target(tile=tile)
+    n = 0
+    for plan in En.restricted_growth(6):
+        if prog.validate(plan, tgt)[0] != 0:
+            continue
+        got, _ = run_kf(desc, plan, inputs, 2, tgt)
+        assert compare(desc, got, ref) == [], plan
+        n += 1
+    assert n == prog.count_legal(tgt) >= 4

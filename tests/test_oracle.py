@@ -441,3 +441,17 @@ def test_resource_model_worked_example():
     assert s["delay"] == {0: 0, 1: 1}
     assert s["smem"] == 6 * 3200 + 4 * 2688 + 16 + 128 == 30096
     assert L.schedule(P.tiny(), [0, 1], L.Target(tile=(32, 16, 0), zunroll=1))["smem"] == 21008
+
+
+def test_L25_radius4_stencil_closed_form_through_stress_program():
+    """Config 5 kernels: L25 (x5040 weights / 5040) of i^2+2j^2+3k^2 is 2+4+6 = 12 exactly in fp64
+    (power-of-two-free but exact: integer weights, products < 2^53), so t1 = 12 and t2 = 0 inside."""
+    prog = P.stress(m=1, n=(20, 20, 20))
+    i, j, k = D.coords(prog)
+    f = (i * i + 2 * j * j + 3 * k * k).astype(np.float64)
+    inp = {"f0": f, "t1_0": np.zeros_like(f), "t2_0": np.zeros_like(f)}
+    out = interp.run(prog, inp, 1)
+    t1 = interior(prog, out["t1_0"])[:, 4:-4, 4:-4]        # away from the periodic xy wrap
+    assert np.allclose(t1, 12.0, rtol=0, atol=1e-9)
+    t2 = interior(prog, out["t2_0"])[4:-4, 8:-8, 8:-8]      # L25 of a constant is 0 (frozen z ghosts differ)
+    assert np.allclose(t2, 0.0, rtol=0, atol=1e-9)

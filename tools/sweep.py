@@ -24,6 +24,8 @@ def main():
             plan = P.weather_hand_plan(desc)
         elif plan_kind == "unfused":
             plan = list(range(44))
+        elif plan_kind.startswith("hgga"):
+            plan, _ = prog.search(kf.SEARCH_HGGA, tgt, seed=1)
         elif plan_kind.startswith("time"):
             plan, _ = prog.search(kf.SEARCH_GREEDY_TIME, tgt)
         else:
