@@ -38,10 +38,13 @@ def workload(name: str):
     from workloads import data, programs
     if name == "weather":
         desc = programs.weather(n=(512, 512, 128))
-        return desc, data.weather_inputs, dict(tile=(64, 4, 0)), "weather-44k31a-512x512x128-fp64 (BASELINE config 3)"
+        return desc, data.weather_inputs, dict(tile=(32, 8, 0)), "weather-44k31a-512x512x128-fp64 (BASELINE config 3)"
     if name == "weather_small":
         desc = programs.weather(n=(128, 128, 64))
         return desc, data.weather_inputs, dict(tile=(32, 16, 0)), "weather-44k31a-128x128x64-fp64"
+    if name == "suite":
+        desc = programs.gen_suite(seed=0)
+        return desc, data.uniform, dict(tile=(32, 8, 0)), "suite-10k8a-256^3-fp32 (BASELINE config 2, gen_suite seed 0)"
     if name == "tiny":
         desc = programs.tiny()
         return desc, data.uniform, dict(tile=(32, 16, 0)), "tiny-3k3a-32^3-fp32 (BASELINE config 1)"
@@ -62,10 +65,10 @@ def choose_plan(prog, target, which: str):
     if which == "hand":
         from workloads.programs import weather_hand_plan
         return weather_hand_plan(prog.desc), "hand plan (App. A.4)"
-    method = kf.SEARCH_BRUTE_TIME if n <= 10 else kf.SEARCH_GREEDY_TIME
-    plan, _ = prog.search(method, target)
+    method = kf.SEARCH_BRUTE_TIME if n <= 10 else kf.SEARCH_HGGA
+    plan, _ = prog.search(method, target, seed=1)
     return plan, ("brute-force on projected time" if method == kf.SEARCH_BRUTE_TIME
-                  else "greedy search on the resource-aware projected time")
+                  else "HGGA search (seed 1) on the resource-aware projected time")
 
 
 # ---------------------------------------------------------------- clocks
@@ -475,7 +478,7 @@ def main():
     ap.add_argument("--impl", default="kf", choices=["kf", "reference"])
     ap.add_argument("--workload", default="weather")
     ap.add_argument("--plan", default="best", choices=["best", "unfused", "hand"])
-    ap.add_argument("--relax-all", type=int, default=1, help="weather: rename every written array (KF_PROG_RELAX_ALL)")
+    ap.add_argument("--relax-all", type=int, default=0, help="weather: rename every written array (KF_PROG_RELAX_ALL)")
     ap.add_argument("--tile", default=None)
     ap.add_argument("--stages", type=int, default=None)
     ap.add_argument("--threads", type=int, default=None)
