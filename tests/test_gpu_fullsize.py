@@ -1,0 +1,73 @@
+"""Parity at BASELINE full size (config 3: weather 512x512x128 fp64) in the launch configuration
+bench.py times (HGGA plan, tile 32x8), checked on sampled windows the oracle computes exactly:
+each window is re-run by the oracle on a crop whose margin covers the step's dependency cone
+(computed from the kernels' footprints), so the window's values are the exact global result."""
+import numpy as np
+import pytest
+
+from oracle import interp
+from workloads import data as D
+from workloads import programs as P
+from workloads.program import BC_FROZEN
+
+from .gpu_util import bits
+
+pytestmark = pytest.mark.gpu
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():
+    pytest.skip("needs a GPU", allow_module_level=True)
+
+import paper_conf_sc_wahibm14_b200 as kf  # noqa: E402
+
+
+def dependency_radius(desc, nsteps):
+    """xy radius of the cone through which an output after `nsteps` depends on the inputs."""
+    rad = {x: 0 for x in range(len(desc.arrays))}
+    for _ in range(nsteps):
+        for kern in desc.kernels:
+            r = max(rad[a] + max(max(abs(d[0]), abs(d[1])) for d in offs) for a, offs in kern.reads().items())
+            for o in kern.writes():
+                rad[o] = max(rad[o], r)
+    return max(rad.values())
+
+
+def crop(desc, arrays, x0, y0, w, margin):
+    """Window [x0, x0+w) x [y0, y0+w) plus margin, wrapped on the periodic xy axes, as a frozen-xy
+    sub-problem (its ghost cells are the true neighbours)."""
+    nx, ny, nz = desc.n
+    g = desc.ghost
+    W = w + 2 * margin
+    xi = (np.arange(-margin - g[0], w + margin + g[0]) + x0) % nx + g[0]
+    yi = (np.arange(-margin - g[1], w + margin + g[1]) + y0) % ny + g[1]
+    sub = desc.with_(n=(W, W, nz), bc=(BC_FROZEN, BC_FROZEN, desc.bc[2]))
+    return sub, {nm: np.ascontiguousarray(a[:, yi][:, :, xi]) for nm, a in arrays.items()}
+
+
+def test_weather_full_size_sampled_windows():
+    desc = P.weather(n=(512, 512, 128))
+    inputs = D.weather_inputs(desc, 3)
+    prog = kf.Program(desc)
+    tgt = kf.Target(tile=(32, 8, 0))
+    plan, _ = prog.search(kf.SEARCH_HGGA, tgt, seed=1)
+    nsteps = 2
+    ex = kf.Exec(prog, plan, tgt)
+    dev = kf.device_arrays(prog, inputs)
+    sb = ex.scratch_bytes()
+    scr = torch.empty(sb, dtype=torch.uint8, device="cuda") if sb else None
+    ex.run(dev, scr, nsteps)
+    torch.cuda.synchronize()
+    got = kf.host_arrays(prog, dev)
+    del dev, scr
+    M = dependency_radius(desc, nsteps) + 1
+    w = 8
+    g = desc.ghost
+    live = [nm for nm in ("DENS", "MOMX", "MOMY", "MOMZ", "RHOT")]
+    for (x0, y0) in ((0, 0), (508, 3), (200, 505), (131, 257)):
+        sub, sin = crop(desc, inputs, x0, y0, w, M)
+        ref = interp.run(sub, sin, nsteps)
+        for nm in live:
+            r = ref[nm][g[2]:g[2] + 128, g[1] + M:g[1] + M + w, g[0] + M:g[0] + M + w]
+            xs = (np.arange(x0, x0 + w) % 512) + g[0]
+            ys = (np.arange(y0, y0 + w) % 512) + g[1]
+            gv = got[nm][g[2]:g[2] + 128][:, ys][:, :, xs]
+            assert np.array_equal(bits(gv), bits(r)), (nm, x0, y0)
