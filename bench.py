@@ -53,7 +53,7 @@ def workload(name: str):
         return desc, data.fig3_inputs, dict(tile=(32, 16, 0)), "fig3-6k-512x512x128-fp64"
     if name == "stress":
         desc = programs.stress(m=2, n=(768, 768, 768))
-        return desc, data.uniform, dict(tile=(32, 16, 0), max_halo=16), "stress-2fields-L25xL25-768^3-fp64 (config 5)"
+        return desc, None, dict(tile=(32, 8, 0), max_halo=16), "stress-2fields-L25xL25-768^3-fp64 (config 5)"
     raise SystemExit(f"unknown workload {name}")
 
 
@@ -305,9 +305,16 @@ def run_kf(args):
         torch.distributed.broadcast(t, 0)
         dist_info = (px, py, rank, world, bytes(t.cpu().tolist()))
     # synthetic inputs of the paper-shaped workload (seed 3 + rank: each rank owns its sub-domain)
-    inputs = gen(desc, 3 + rank)
-    dev = kf.device_arrays(prog, inputs)
-    del inputs
+    if gen is None:
+        # large uniform workloads: U[-1,1) generated on the device (seeded torch generator)
+        L = prog.layout()
+        gdev = torch.Generator(device="cuda").manual_seed(3 + rank)
+        dt = torch.float64 if desc.dtype == 1 else torch.float32
+        dev = [torch.rand(L.elems, generator=gdev, device="cuda", dtype=dt) * 2 - 1 for _ in desc.arrays]
+    else:
+        inputs = gen(desc, 3 + rank)
+        dev = kf.device_arrays(prog, inputs)
+        del inputs
     stream = torch.cuda.current_stream()
     t0 = time.time()
     tuned, gtargets = None, None
@@ -340,7 +347,7 @@ def run_kf(args):
         del rn_u
     # end-to-end through the public API with host buffers (copies inside the timed region)
     e2e = None
-    if not args.no_e2e:
+    if not args.no_e2e and gen is not None:
         k = max(1, min(args.steps, 3))
         if rn.dist is None:
             host = [t.cpu().pin_memory() for t in dev]
