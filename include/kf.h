@@ -165,8 +165,10 @@ typedef struct {
   int32_t internal_axes;         /* bitmask of axes split across ranks (V6 treats as wrap) */
   int32_t zunroll;               /* planes per stream iteration U in [1,4] (ILP; ring depth) */
   int32_t pblock[2];             /* points per thread in x, y (register blocking), [1,4] each */
+  int32_t ringunroll;            /* 1: ring sizes rounded to powers of two and the stream loop
+                                    unrolled so every SMEM slot is a compile-time constant    */
 } kf_target;
-/* Fills the B200 defaults: 8.0e12, 232448, 255, 148, {64,4,0}, 2, 256, 16, 0, 1, {1,1}. */
+/* Fills the B200 defaults: 8.0e12, 232448, 255, 148, {64,4,0}, 2, 256, 16, 0, 1, {1,1}, 0. */
 kf_status kf_target_b200(kf_target* out);
 
 /* ------------------------------------------------------------------ legality (Eq. 1.1-1.7) */

@@ -43,6 +43,7 @@ class Target:
     internal_axes: int = 0          # bitmask of axes split across ranks (treated like periodic by V6)
     zunroll: int = 1                # planes per stream iteration U (ring depth grows with U, R20)
     pblock: Tuple[int, int] = (1, 1)  # points per thread in x, y (register blocking)
+    ringunroll: int = 0             # 1: ring depths rounded up to powers of two (R20b)
 
 
 # ---------------------------------------------------------------- plans
@@ -221,6 +222,8 @@ def schedule(prog: Program, grp: List[int], target: Target):
             span = max(D[c] - d[2] for c, offs in rd for d in offs) - D[p] + 1 + (target.zunroll - 1)
             (lo, hi) = ext[p]
             res.append(("mid", x, v, TX + lo[0] + hi[0], TY + lo[1] + hi[1], span, 0, 0))
+    if target.ringunroll:   # ring depths rounded up to powers of two (stream loop unrolled, R20b)
+        res = [r[:5] + (1 << (r[5] - 1).bit_length(),) + r[6:] for r in res]
     smem = 0
     for r in res:
         px = _roundup(r[3], 16 // es)

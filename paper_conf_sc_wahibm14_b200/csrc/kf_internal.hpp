@@ -126,6 +126,7 @@ struct GroupLowering {
   int tile[3];
   int stages = 2, threads = 256, zunroll = 1;
   int pblock[2] = {1, 1};   // points per thread in x, y (register blocking in the fast path)
+  int ring_unroll = 0;      // 0, or N: every ring size a power of two dividing N, loop unrolled N times
   int ring_of(const Ver& v) const;        // index in rings or -1
 };
 

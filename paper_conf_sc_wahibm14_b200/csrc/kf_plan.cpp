@@ -194,6 +194,17 @@ GroupLowering lower_group(const Program& p, const std::vector<int>& g, const kf_
       finish_ring(r);
       L.rings.push_back(r);
     }
+  // ring unrolling (target.ringunroll): sizes rounded up to powers of two; N = the largest (<= 16)
+  if (t.ringunroll) {
+    int N = 1;
+    for (auto& r : L.rings) {
+      int q = 1;
+      while (q < r.slots) q *= 2;
+      r.slots = q;
+      N = std::max(N, q);
+    }
+    L.ring_unroll = N <= 16 ? N : 0;
+  }
   // ---- SMEM layout and the resource model (R20)
   int off = 0;
   for (auto& r : L.rings) {
@@ -442,6 +453,7 @@ void check_target(const kf_target* t) {
   if (t->tile[0] % 4) fail(KF_E_ARG, "tile TX must be a multiple of 4 (16-byte aligned TMA boxes)");
   if (t->stages < 2 || t->stages > 8) fail(KF_E_ARG, "stages must be in [2, 8]");
   if (t->zunroll < 1 || t->zunroll > 4) fail(KF_E_ARG, "zunroll must be in [1, 4]");
+  if (t->ringunroll < 0 || t->ringunroll > 1) fail(KF_E_ARG, "ringunroll must be 0 or 1");
   if (t->pblock[0] < 1 || t->pblock[0] > 4 || t->pblock[1] < 1 || t->pblock[1] > 4)
     fail(KF_E_ARG, "pblock must be in [1, 4] x [1, 4]");
   if (t->threads < 32 || t->threads > 1024 || t->threads % 32) fail(KF_E_ARG, "threads must be a multiple of 32 in [32,1024]");

@@ -344,6 +344,7 @@ kf_status kf_target_b200(kf_target* out) {
     t.zunroll = 1;
     t.pblock[0] = 1;
     t.pblock[1] = 1;
+    t.ringunroll = 0;
     *out = t;
   });
 }

@@ -124,7 +124,8 @@ def test_resource_limits_V7_V8():
     for zu in (1, 3):
         check_program(desc, target=(L.Target(zunroll=zu, tile=(16, 8, 0)), kf.Target(zunroll=zu, tile=(16, 8, 0))))
     for kw in (dict(pblock=(2, 2), zunroll=2, threads=128, tile=(32, 8, 0)), dict(pblock=(1, 3), threads=64, tile=(16, 16, 0)),
-               dict(pblock=(4, 1), threads=32, tile=(64, 4, 0))):
+               dict(pblock=(4, 1), threads=32, tile=(64, 4, 0)), dict(ringunroll=1, zunroll=2, tile=(32, 8, 0)),
+               dict(ringunroll=1, tile=(16, 16, 0), stages=3)):
         check_program(P.fig3(), target=(L.Target(**kw), kf.Target(**kw)))
     tk = kf.Target(regs_per_thread_max=40, zunroll=2)
     to = L.Target(regs_per_thread_max=40, zunroll=2)

@@ -47,11 +47,12 @@ def test_tiny_closed_form_on_gpu():
 
 @pytest.mark.parametrize("tile", [(32, 16, 0), (16, 8, 0), (32, 16, 7), (8, 8, 5)])
 @pytest.mark.parametrize("zunroll", [1, 2, 3])
-def test_tiny_ragged_tiles_and_z_chunks(tile, zunroll):
+@pytest.mark.parametrize("ringunroll", [0, 1])
+def test_tiny_ragged_tiles_and_z_chunks(tile, zunroll, ringunroll):
     desc = P.tiny(n=(37, 21, 19))
     inputs = D.uniform(desc, 2)
     ref = interp.run(desc, inputs, 3)
-    got, _ = run_kf(desc, [0, 0, 1], inputs, 3, kf.Target(tile=tile, zunroll=zunroll))
+    got, _ = run_kf(desc, [0, 0, 1], inputs, 3, kf.Target(tile=tile, zunroll=zunroll, ringunroll=ringunroll))
     assert compare(desc, got, ref) == []
 
 
@@ -83,8 +84,9 @@ def test_random_programs_random_legal_plans(seed):
     tile = [(32, 16, 0), (16, 16, 0), (8, 4, 6), (32, 8, 11)][seed % 4]
     zu = [1, 2, 3][seed % 3]
     pb = [(1, 1), (2, 1), (2, 2), (1, 3)][seed % 4]
+    ru = seed % 2
     for plan in pick:
-        got, _ = run_kf(desc, plan, inputs, nsteps, kf.Target(tile=tile, zunroll=zu, pblock=pb, threads=64))
+        got, _ = run_kf(desc, plan, inputs, nsteps, kf.Target(tile=tile, zunroll=zu, pblock=pb, threads=64, ringunroll=ru))
         assert compare(desc, got, ref) == [], (plan, tile)
 
 
@@ -96,9 +98,9 @@ def test_weather_small_fp64_plans():
     ref = interp.run(desc, inputs, 2)
     plan_g, _ = kf.Program(desc).search(kf.SEARCH_GREEDY, kf.Target(tile=(32, 8, 0), zunroll=2))
     for plan in (list(range(44)), weather_hand_plan(desc), plan_g):
-        for zu in (1, 2):
-            got, _ = run_kf(desc, plan, inputs, 2, kf.Target(tile=(32, 8, 0), zunroll=zu))
-            assert compare(desc, got, ref) == [], (plan, zu)
+        for zu, ru in ((1, 0), (2, 0), (1, 1)):
+            got, _ = run_kf(desc, plan, inputs, 2, kf.Target(tile=(32, 8, 0), zunroll=zu, ringunroll=ru))
+            assert compare(desc, got, ref) == [], (plan, zu, ru)
 
 
 def test_graph_and_eager_agree_and_odd_even_steps():
