@@ -177,8 +177,9 @@ def cpu_baseline(name: str, budget_s: float = 12.0):
 
 
 # ---------------------------------------------------------------- GPU timing
-AUTOTUNE_CANDIDATES = [((64, 4, 0), 2, 1), ((64, 4, 0), 2, 2), ((32, 8, 0), 2, 1), ((32, 8, 0), 2, 2),
-                       ((64, 4, 0), 3, 1), ((32, 8, 0), 3, 1), ((32, 4, 0), 2, 1), ((64, 8, 0), 2, 1)]
+AUTOTUNE_CANDIDATES = [((64, 4, 0), 2, 1, 0), ((64, 4, 0), 2, 2, 0), ((32, 8, 0), 2, 1, 0), ((32, 8, 0), 2, 2, 0),
+                       ((64, 4, 0), 3, 1, 0), ((32, 8, 0), 3, 1, 0), ((32, 4, 0), 2, 1, 0), ((64, 8, 0), 2, 1, 0),
+                       ((32, 8, 0), 2, 1, 1), ((64, 4, 0), 2, 1, 1), ((32, 8, 0), 2, 2, 1)]
 
 
 def autotune(prog, plan, dev, base_kw, steps=4):
@@ -189,9 +190,9 @@ def autotune(prog, plan, dev, base_kw, steps=4):
     import paper_conf_sc_wahibm14_b200 as kf
     best = None
     tried = []
-    for tile, stages, zu in AUTOTUNE_CANDIDATES:
+    for tile, stages, zu, ru in AUTOTUNE_CANDIDATES:
         kw = dict(base_kw)
-        kw.update(tile=tile, stages=stages, zunroll=zu)
+        kw.update(tile=tile, stages=stages, zunroll=zu, ringunroll=ru)
         tgt = kf.Target(**kw)
         try:
             ex = kf.Exec(prog, plan, tgt)
@@ -205,13 +206,14 @@ def autotune(prog, plan, dev, base_kw, steps=4):
         ex.run(dev, scr, steps)
         torch.cuda.synchronize()
         gms, _ = ex.group_times()
-        tried.append(((tile, stages, zu), [g / steps for g in gms]))
+        tried.append(((tile, stages, zu, ru), [g / steps for g in gms]))
         if best is None:
             best = [(g / steps, kw) for g in gms]
         else:
             best = [min(b, (g / steps, kw), key=lambda v: v[0]) for b, g in zip(best, gms)]
         del ex, scr
-    return [kf.Target(**kw) for _, kw in best], [(list(kw["tile"]), kw["stages"], kw["zunroll"]) for _, kw in best], tried
+    return ([kf.Target(**kw) for _, kw in best],
+            [(list(kw["tile"]), kw["stages"], kw["zunroll"], kw["ringunroll"]) for _, kw in best], tried)
 
 
 def max_over_ranks(x: float) -> float:
@@ -325,7 +327,8 @@ def run_kf(args):
             obj = [tuned]
             torch.distributed.broadcast_object_list(obj, 0)
             tuned = obj[0]
-            gtargets = [kf.Target(**dict(tkw, tile=tuple(c[0]), stages=c[1], zunroll=c[2])) for c in tuned]
+            gtargets = [kf.Target(**dict(tkw, tile=tuple(c[0]), stages=c[1], zunroll=c[2], ringunroll=c[3]))
+                        for c in tuned]
     rn = Runner(prog, plan, target, gtargets, dist_info)
     jit_s = time.time() - t0
     info = rn.ex.info()

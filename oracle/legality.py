@@ -243,7 +243,7 @@ def schedule(prog: Program, grp: List[int], target: Target):
         nb = (-(-w // bx)) * (-(-h // by))
         rounds = max(rounds, -(-nb // threads))
     P = min(8, target.pblock[0] * target.pblock[1] * target.zunroll * rounds)
-    regs = 32 + 2 * (es // 4) * (depth + 3) * P
+    regs = 48 + 2 * (es // 4) * (depth + 3) * P
     return dict(ext=ext, pts=pts, delay=D, res=res, smem=smem, regs=regs, alive=alive)
 
 

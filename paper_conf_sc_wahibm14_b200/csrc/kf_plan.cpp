@@ -239,7 +239,7 @@ GroupLowering lower_group(const Program& p, const std::vector<int>& g, const kf_
     rounds = std::max(rounds, (nb + L.threads - 1) / L.threads);
   }
   const int P = std::min(8, t.pblock[0] * t.pblock[1] * U * rounds);
-  L.regs = 32 + 2 * (es / 4) * (depth + 3) * P;
+  L.regs = 48 + 2 * (es / 4) * (depth + 3) * P;
   return L;
 }
 
