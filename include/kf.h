@@ -222,6 +222,21 @@ typedef struct { int32_t kernel, alive, delay, pad; int32_t elo[3], ehi[3]; } kf
 kf_status kf_group_schedule(const kf_program* prog, const int32_t* plan, const kf_target* target,
                             int32_t group, kf_kernel_sched* out, int32_t cap, int32_t* n);
 
+/* The paper's own projection for one new kernel (Eq. 2-10) from Table III/IV
+ * metadata, as printed (readings R11-R14: Hal in points, "8" = element bytes).  Reproduces the
+ * worked example of P:372 (B_Sh = 688, P_MemBound = 29.688 GFLOPS); the B200 search uses
+ * kf_group_proj.t_model_s instead (R22). */
+typedef struct {
+  int32_t t_b, blocks_smx, thr, blocks, hal, halo, shared_arrays, smx;   /* T_B, Blocks_SMX, Thr, B, Hal, c, |ShrLst|, #SMX */
+  int32_t r_t, r_max, r_smx, r_adr, sh_smx, b_conf, elem_bytes, pad;      /* R_T, R_Max, R_SMX (regs), R_Adr, Sh_SMX (B), B_conf (B) */
+  double gmem_bw_gbs, regfac, max_thread_load, fl_unfused_sum, flop_halo_sum;
+} kf_paper_meta;
+typedef struct {
+  int32_t h_th, eq2_ok, eq3_ok, eq6_ok, eq7_ok, pad;
+  double b_sh, b_eff, p_membound_gflops, t_pro_s;
+} kf_paper_proj;
+kf_status kf_paper_projection(const kf_paper_meta* meta, kf_paper_proj* out);
+
 /* ------------------------------------------------------------------ plan search */
 typedef enum {
   KF_SEARCH_BRUTE = 0,   /* all restricted-growth strings with pruning (n <= 14)           */

@@ -94,6 +94,17 @@ class kf_group_info(C.Structure):
                 ("bytes_per_launch", C.c_uint64), ("name", C.c_char * 64)]
 
 
+class kf_paper_meta(C.Structure):
+    _fields_ = [(n, C.c_int32) for n in ("t_b", "blocks_smx", "thr", "blocks", "hal", "halo", "shared_arrays", "smx",
+                                         "r_t", "r_max", "r_smx", "r_adr", "sh_smx", "b_conf", "elem_bytes", "pad")] + \
+               [(n, C.c_double) for n in ("gmem_bw_gbs", "regfac", "max_thread_load", "fl_unfused_sum", "flop_halo_sum")]
+
+
+class kf_paper_proj(C.Structure):
+    _fields_ = [(n, C.c_int32) for n in ("h_th", "eq2_ok", "eq3_ok", "eq6_ok", "eq7_ok", "pad")] + \
+               [(n, C.c_double) for n in ("b_sh", "b_eff", "p_membound_gflops", "t_pro_s")]
+
+
 P = C.c_void_p
 I32P = C.POINTER(C.c_int32)
 U64P = C.POINTER(C.c_uint64)
@@ -132,6 +143,7 @@ SIGNATURES = {
     "kf_exec_group_times": (C.c_int, [P, C.POINTER(C.c_double), C.c_int32, I32P, C.POINTER(C.c_int64)]),
     "kf_exec_set_graph": (C.c_int, [P, C.c_int32]),
     "kf_flush_l2": (C.c_int, [P, C.c_uint64, P]),
+    "kf_paper_projection": (C.c_int, [C.POINTER(kf_paper_meta), C.POINTER(kf_paper_proj)]),
     "kf_dist_unique_id": (C.c_int, [C.POINTER(C.c_uint8)]),
     "kf_dist_neighbors": (C.c_int, [C.c_int32, C.c_int32, C.c_int32, I32P]),
     "kf_dist_create": (C.c_int, [C.POINTER(P), C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.c_int32,

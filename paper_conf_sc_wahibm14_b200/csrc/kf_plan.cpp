@@ -583,3 +583,32 @@ kf_status kf_group_schedule(const kf_program* prog, const int32_t* plan, const k
 }
 
 }  // extern "C"
+
+// ---------------------------------------------------------------- paper Eq. 2-10 (NEXT-2)
+// The paper's codeless upper-bound projection for one new kernel, evaluated from
+// the Table III / Table IV metadata exactly as printed.  Used to reproduce the worked example
+// (B_Sh = 688, P_MemBound = 29.688 GFLOPS); not the B200 search objective (R22).
+extern "C" kf_status kf_paper_projection(const kf_paper_meta* m, kf_paper_proj* out) {
+  KF_TRY({
+    if (!m || !out) fail(KF_E_ARG, "null argument");
+    if (m->thr <= 0 || m->blocks <= 0 || m->shared_arrays <= 0 || m->gmem_bw_gbs <= 0 || m->elem_bytes <= 0)
+      fail(KF_E_ARG, "thr, blocks, shared_arrays, gmem_bw_gbs, elem_bytes must be > 0");
+    kf_paper_proj r{};
+    const int c = m->halo ? 1 : 0;
+    r.h_th = (m->hal + m->thr - 1) / m->thr;                                   // H_TH = ceil(Hal/Thr)
+    const double denom = double(1 + c * r.h_th) * m->shared_arrays;
+    r.b_sh = double(m->t_b) * m->blocks_smx / denom;                            // Eq. 8
+    r.b_eff = r.b_sh * m->smx / (double(m->thr) * m->blocks);                   // B_eff
+    r.p_membound_gflops = r.b_eff * m->gmem_bw_gbs / m->elem_bytes;             // Eq. 9 ("8" = fp64 bytes, R14)
+    const double flops = m->fl_unfused_sum + m->flop_halo_sum * m->hal / (double(m->blocks) * m->thr);
+    r.t_pro_s = flops * 1e-9 / r.p_membound_gflops;                             // Eq. 10 (R12)
+    // constraints
+    const double regs_blocking = m->regfac * m->max_thread_load + c * r.h_th + 1;   // Eq. 4 lower bound
+    const double r_fetch = 1 + c * r.h_th;                                          // Eq. 5
+    r.eq2_ok = m->r_t <= m->r_max;
+    r.eq3_ok = double(m->blocks_smx) * m->thr * m->r_t <= m->r_smx;
+    r.eq6_ok = r_fetch + regs_blocking + m->r_adr < m->r_t && m->r_t <= m->r_max;
+    r.eq7_ok = double(1 + c * r.h_th) * m->t_b * m->blocks_smx * m->shared_arrays * m->elem_bytes + m->b_conf <= m->sh_smx;
+    *out = r;
+  });
+}

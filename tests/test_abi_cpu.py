@@ -209,3 +209,24 @@ def test_hgga_weather_no_worse_than_greedy():
     th = sum(g.t_model_s for g in p.project(plan_h)[0])
     tg = sum(g.t_model_s for g in p.project(plan_g)[0])
     assert th <= tg * 1.0001
+
+
+def test_paper_projection_abi_matches_oracle_and_example():
+    import ctypes
+    import json
+    import os
+    from oracle import paper_model
+    from paper_conf_sc_wahibm14_b200._abi import kf_paper_meta, kf_paper_proj, lib
+    gold = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "eq8_worked_example.json")))["inputs"]
+    m = kf_paper_meta()
+    for k, v in gold.items():
+        setattr(m, k, v)
+    m.fl_unfused_sum, m.flop_halo_sum = 3.2e9, 1.1e6
+    m.r_t, m.r_max, m.r_smx, m.r_adr, m.sh_smx, m.regfac, m.max_thread_load = 40, 255, 65536, 4, 49152, 0.85, 3
+    out = kf_paper_proj()
+    assert lib().kf_paper_projection(ctypes.byref(m), ctypes.byref(out)) == 0
+    ref = paper_model.project(**gold, fl_unfused_sum=3.2e9, flop_halo_sum=1.1e6)
+    assert out.b_sh == 688 == ref["b_sh"]
+    assert out.p_membound_gflops == ref["p_membound_gflops"]
+    assert out.t_pro_s == ref["t_pro_s"]
+    assert out.eq2_ok and out.eq3_ok is not None

@@ -455,3 +455,15 @@ def test_L25_radius4_stencil_closed_form_through_stress_program():
     assert np.allclose(t1, 12.0, rtol=0, atol=1e-9)
     t2 = interior(prog, out["t2_0"])[4:-4, 8:-8, 8:-8]      # L25 of a constant is 0 (frozen z ghosts differ)
     assert np.allclose(t2, 0.0, rtol=0, atol=1e-9)
+
+
+def test_paper_eq8_worked_example_golden():
+    """NEXT-2 pin: the paper's worked example: B_Sh = 688 exactly, and the printed
+    formula 688*14*202/(8*128*64) = 29.688 GFLOPS (75.37 % of 39.39; the paper prints 75.8 %)."""
+    from oracle import paper_model
+    gold = json.load(open(os.path.join(GOLD, "eq8_worked_example.json")))
+    r = paper_model.project(**gold["inputs"])
+    assert r["h_th"] == 1
+    assert r["b_sh"] == gold["printed"]["b_sh"]
+    assert r["p_membound_gflops"] == 688 * 14 * 202 / (8 * 128 * 64) == gold["derived_from_printed_formula"]["p_membound_gflops"]
+    assert round(100 * r["p_membound_gflops"] / gold["printed"]["roofline_gflops"], 2) == gold["derived_from_printed_formula"]["percent"]
