@@ -127,6 +127,7 @@ struct GroupLowering {
   int stages = 2, threads = 256, zunroll = 1;
   int pblock[2] = {1, 1};   // points per thread in x, y (register blocking in the fast path)
   int ring_unroll = 0;      // 0, or N: every ring size a power of two dividing N, loop unrolled N times
+  bool ghost_write = false; // live-out stores also write the periodic x/y ghost copies (no fills)
   int ring_of(const Ver& v) const;        // index in rings or -1
 };
 

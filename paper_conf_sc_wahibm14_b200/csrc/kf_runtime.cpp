@@ -164,7 +164,8 @@ struct kf_exec {
   std::vector<int> order;
   std::vector<GroupExec> G;
   int period = 1;
-  std::vector<std::vector<Op>> sched;      // per parity
+  std::vector<std::vector<Op>> sched;      // per parity (fills dropped when groups write ghost copies)
+  std::vector<std::vector<Op>> sched_full; // per parity, every fill (domain decomposition exchanges)
   std::vector<Ver> scratch_vers;           // scratch buffer i holds (x, v)
   uint64_t scratch_bytes = 0, array_bytes = 0;
   std::vector<int> fill_all;               // buffers filled once at the start of a run
@@ -391,6 +392,18 @@ static void build_schedule(kf_exec* E) {
     for (int par = 0; par < E->period; par++)
       for (const GroupExec& g : E->G)
         for (const Ver& v : g.mids) all_fill.insert(buffer_id(E, v, par));
+  E->sched_full = sched;
+  // when every group writes periodic ghost copies with its live-out stores, buffers are never
+  // dirty: drop the in-loop fills (the one-time fills at run start stay)
+  bool all_gw = true;
+  for (const GroupExec& g : E->G) all_gw = all_gw && g.L.ghost_write;
+  if (all_gw)
+    for (auto& ops : sched) {
+      std::vector<Op> k;
+      for (const Op& op : ops)
+        if (op.kind != 0) k.push_back(op);
+      ops = k;
+    }
   E->sched = sched;
   E->fill_all.assign(all_fill.begin(), all_fill.end());
 }
@@ -934,7 +947,7 @@ static void dist_run(kf_dist* D, void* const* arrays, void* const* scratch, uint
   for (int b : E0->fill_all) dist_exchange(D, b, s);
   for (int64_t step = 0; step < nsteps; step++) {
     const int par = int(step % E0->period);
-    for (const Op& op : E0->sched[par]) {
+    for (const Op& op : E0->sched_full[par]) {
       if (op.kind == 0) {
         dist_exchange(D, op.buf, s);
       } else {
