@@ -170,7 +170,7 @@ typedef struct {
   int32_t ghostwrite;            /* 1: stores also write periodic x/y ghost copies, so the step
                                     needs no ghost-fill kernels (single-domain runs)          */
 } kf_target;
-/* Fills the B200 defaults: 8.0e12, 232448, 255, 148, {64,4,0}, 2, 256, 16, 0, 1, {1,1}, 0, 1. */
+/* Fills the B200 defaults: 8.0e12, 232448, 255, 148, {64,4,0}, 2, 256, 16, 0, 1, {1,1}, 0, 0. */
 kf_status kf_target_b200(kf_target* out);
 
 /* ------------------------------------------------------------------ legality (Eq. 1.1-1.7) */

@@ -85,8 +85,10 @@ def test_random_programs_random_legal_plans(seed):
     zu = [1, 2, 3][seed % 3]
     pb = [(1, 1), (2, 1), (2, 2), (1, 3)][seed % 4]
     ru = seed % 2
+    gw = (seed // 2) % 2
     for plan in pick:
-        got, _ = run_kf(desc, plan, inputs, nsteps, kf.Target(tile=tile, zunroll=zu, pblock=pb, threads=64, ringunroll=ru))
+        got, _ = run_kf(desc, plan, inputs, nsteps, kf.Target(tile=tile, zunroll=zu, pblock=pb, threads=64, ringunroll=ru,
+                                                              ghostwrite=gw))
         assert compare(desc, got, ref) == [], (plan, tile)
 
 
@@ -98,8 +100,8 @@ def test_weather_small_fp64_plans():
     ref = interp.run(desc, inputs, 2)
     plan_g, _ = kf.Program(desc).search(kf.SEARCH_GREEDY, kf.Target(tile=(32, 8, 0), zunroll=2))
     for plan in (list(range(44)), weather_hand_plan(desc), plan_g):
-        for zu, ru in ((1, 0), (2, 0), (1, 1)):
-            got, _ = run_kf(desc, plan, inputs, 2, kf.Target(tile=(32, 8, 0), zunroll=zu, ringunroll=ru))
+        for zu, ru, gw in ((1, 0, 1), (2, 0, 0), (1, 1, 1)):
+            got, _ = run_kf(desc, plan, inputs, 2, kf.Target(tile=(32, 8, 0), zunroll=zu, ringunroll=ru, ghostwrite=gw))
             assert compare(desc, got, ref) == [], (plan, zu, ru)
 
 
