@@ -177,9 +177,10 @@ def cpu_baseline(name: str, budget_s: float = 12.0):
 
 
 # ---------------------------------------------------------------- GPU timing
-AUTOTUNE_CANDIDATES = [((64, 4, 0), 2, 1, 0), ((64, 4, 0), 2, 2, 0), ((32, 8, 0), 2, 1, 0), ((32, 8, 0), 2, 2, 0),
-                       ((64, 4, 0), 3, 1, 0), ((32, 8, 0), 3, 1, 0), ((32, 4, 0), 2, 1, 0), ((64, 8, 0), 2, 1, 0),
-                       ((32, 8, 0), 2, 1, 1), ((64, 4, 0), 2, 1, 1), ((32, 8, 0), 2, 2, 1)]
+AUTOTUNE_CANDIDATES = [((32, 8, 0), 2, 1, 0), ((32, 8, 64), 2, 1, 0), ((32, 8, 32), 2, 1, 0), ((64, 4, 0), 2, 1, 0),
+                       ((64, 4, 64), 2, 1, 0), ((64, 8, 0), 2, 1, 0), ((64, 8, 64), 2, 1, 0), ((32, 8, 64), 2, 2, 0),
+                       ((64, 4, 0), 2, 2, 0), ((32, 8, 0), 3, 1, 0), ((32, 8, 64), 2, 1, 1), ((64, 4, 64), 2, 1, 1),
+                       ((32, 8, 64), 2, 2, 1)]
 
 
 def autotune(prog, plan, dev, base_kw, steps=4):
@@ -320,7 +321,11 @@ def run_kf(args):
     stream = torch.cuda.current_stream()
     t0 = time.time()
     tuned, gtargets = None, None
-    if args.autotune:
+    if args.tuned:   # fixed per-group configs (e.g. for an ncu run of exactly the timed configuration)
+        tuned = json.loads(args.tuned)
+        gtargets = [kf.Target(**dict(tkw, tile=tuple(c[0]), stages=c[1], zunroll=c[2], ringunroll=c[3]))
+                    for c in tuned]
+    elif args.autotune:
         if rank == 0:
             gtargets, tuned, _ = autotune(prog, plan, dev, tkw)
         if world > 1:
@@ -496,6 +501,8 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--autotune", type=int, default=1, help="per-group launch configuration by measurement (1/0)")
+    ap.add_argument("--tuned", default=None, help="JSON per-group configs [[tile,stages,zunroll,ringunroll],...] "
+                                                  "(skips autotune; as printed in config.per_group_launch_config)")
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "kf":
         args.warmup = 3

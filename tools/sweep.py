@@ -20,7 +20,9 @@ def main():
         zu = cfg[3] if len(cfg) > 3 else 1
         pb = cfg[4] if len(cfg) > 4 else [1, 1]
         ru = cfg[5] if len(cfg) > 5 else 0
-        gw = cfg[6] if len(cfg) > 6 else 1
+        gw = cfg[6] if len(cfg) > 6 else 0
+        if len(cfg) > 7:   # codegen A/B knob: max z-queue registers per thread
+            os.environ["KF_ZQ_MAX"] = str(cfg[7])
         tgt = kf.Target(tile=tile, stages=stages, threads=threads, zunroll=zu, pblock=pb, ringunroll=ru, ghostwrite=gw)
         if plan_kind == "hand":
             plan = P.weather_hand_plan(desc)
@@ -51,7 +53,7 @@ def main():
         gms, _ = ex.group_times()
         info = ex.info()
         per, _, _ = prog.project(plan, tgt)
-        r = {"plan": plan_kind, "model_ms": sum(g.t_model_s for g in per) * 1e3, "tile": tile, "stages": stages, "threads": threads, "zunroll": zu, "pblock": pb, "ringunroll": ru, "ghostwrite": gw, "hoist": bool(os.environ.get("KF_HOIST_PTRS")), "ms_per_step": ms,
+        r = {"plan": plan_kind, "model_ms": sum(g.t_model_s for g in per) * 1e3, "tile": tile, "stages": stages, "threads": threads, "zunroll": zu, "pblock": pb, "ringunroll": ru, "ghostwrite": gw, "zq_max": os.environ.get("KF_ZQ_MAX"), "ms_per_step": ms,
              "TBps": info.compulsory_bytes_per_step / ms / 1e9,
              "groups": [(ex.group_info(g).name.decode(), round(gms[g] / 10, 4),
                          round(ex.group_info(g).bytes_per_launch / (gms[g] / 10) / 1e9, 2),
