@@ -231,12 +231,18 @@ def schedule(prog: Program, grp: List[int], target: Target):
         smem += r[5] * plane
     smem += 8 * S + 128
     depth = max([rpn_depth(s.rpn) for k in grp for s in prog.kernels[k].stmts] + [1])
-    # threads per CTA: cover the largest extended region in one pass when the tile has at most one
-    # point per thread (<= 512); points per thread P = pblock x zunroll x rounds (capped at 8)
+    # threads per CTA: one per register block (bx x by points) of the canvas when
+    # the tile's blocks fit the target's thread count (<= 512); points per thread
+    # P = pblock x zunroll x rounds (capped at 8)
     regions = [((TX + ext[k][0][0] + ext[k][1][0]), (TY + ext[k][0][1] + ext[k][1][1])) for k in alive]
-    maxr = max([w * h for w, h in regions] + [0])
-    nt = _roundup(maxr, 32)
-    threads = nt if (TX * TY <= target.threads and target.threads < nt <= 512) else target.threads
+    bx0, by0 = max(1, target.pblock[0]), max(1, target.pblock[1])
+    # canvas = bounding box of all extended regions (per-axis max lo / max hi halo)
+    cw = TX + max([ext[k][0][0] for k in alive] + [0]) + max([ext[k][1][0] for k in alive] + [0])
+    ch = TY + max([ext[k][0][1] for k in alive] + [0]) + max([ext[k][1][1] for k in alive] + [0])
+    maxb = (-(-cw // min(bx0, cw))) * (-(-ch // min(by0, ch))) if alive else 0
+    nt = _roundup(maxb, 32)
+    tb = (-(-TX // bx0)) * (-(-TY // by0))
+    threads = nt if (tb <= target.threads and 32 <= nt <= 512) else target.threads
     rounds = 1
     for w, h in regions:
         bx, by = min(target.pblock[0], w), min(target.pblock[1], h)

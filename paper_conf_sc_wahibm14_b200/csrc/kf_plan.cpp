@@ -217,18 +217,25 @@ GroupLowering lower_group(const Program& p, const std::vector<int>& g, const kf_
   }
   L.mbar_off = off;
   L.smem = off + 8 * S + 128;
-  // threads per CTA: enough to cover the largest extended region in one pass (a region just
-  // above the thread count would otherwise take a second, nearly empty round), within [threads, 512]
+  // threads per CTA: one per register block (bx x by points, pblock) of the largest extended
+  // region, so the fast path covers every region in one pass without clamped duplicate lanes
+  // (which would still issue shared loads); used when the tile itself fits the target's thread
+  // count, capped at 512 (R20)
   {
-    int maxr = 0;
-    for (int k : alive) {
-      const Ext& e = L.ext[k];
-      maxr = std::max(maxr, (TX + e.elo[0] + e.ehi[0]) * (TY + e.elo[1] + e.ehi[1]));
-    }
-    int nt = (maxr + 31) / 32 * 32;
-    // only when the tile itself has at most one point per thread; otherwise the unrolled
-    // rounds of the fast path absorb the halo (critical path P+1 rounds instead of P)
-    L.threads = (t.tile[0] * t.tile[1] <= t.threads && nt > t.threads && nt <= 512) ? nt : t.threads;
+    // the canvas = bounding box of all extended regions (per-axis max lo/hi halo): the fast path
+    // gives each canvas point to one thread for every kernel of the group
+    const int bx = std::max(1, t.pblock[0]), by = std::max(1, t.pblock[1]);
+    int clo[2] = {0, 0}, chi[2] = {0, 0};
+    for (int k : alive)
+      for (int a = 0; a < 2; a++) {
+        clo[a] = std::max(clo[a], L.ext[k].elo[a]);
+        chi[a] = std::max(chi[a], L.ext[k].ehi[a]);
+      }
+    const int CW = TX + clo[0] + chi[0], CH = TY + clo[1] + chi[1];
+    const int maxb = alive.empty() ? 0 : ((CW + std::min(bx, CW) - 1) / std::min(bx, CW)) * ((CH + std::min(by, CH) - 1) / std::min(by, CH));
+    const int nt = (maxb + 31) / 32 * 32;
+    const int tb = ((TX + bx - 1) / bx) * ((TY + by - 1) / by);
+    L.threads = (tb <= t.threads && nt >= 32 && nt <= 512) ? nt : t.threads;
   }
   int depth = 1;
   for (int k : g) depth = std::max(depth, p.kernels[k].depth);
