@@ -4,6 +4,7 @@
 #pragma once
 
 #include <array>
+#include <cstdlib>
 #include <cstdint>
 #include <map>
 #include <memory>
@@ -151,6 +152,30 @@ uint64_t group_bytes(const Program& p, const std::vector<int>& g, uint64_t* rd, 
 // Resource-aware projected time of one fused group (NEXT-2 direction, R22): HBM time of the
 // compulsory bytes at the achievable copy rate, plus issue time of the recomputed regions.
 double model_time(const Program& p, const GroupLowering& L, const kf_target& t, uint64_t bytes);
+
+// ---------------------------------------------------------------- canvas (fast iterations)
+// The fast iterations of a group kernel give each point of the canvas (bounding box of all
+// extended regions) to one thread for every kernel; reads at xy offset 0 of a plane computed in
+// the same iteration are forwarded in registers and identical shared loads are issued once.
+struct CanvasKey {
+  int ring, po, off;   // ring, plane offset from the stream position t, element offset from the canvas point
+  bool operator<(const CanvasKey& o) const {
+    return ring != o.ring ? ring < o.ring : po != o.po ? po < o.po : off < o.off;
+  }
+};
+using Rect = std::array<int, 4>;   // canvas x0, x1, y0, y1 (half open)
+struct CanvasPlan {
+  bool ok = false;                 // one canvas point per thread (else the per-kernel fast path)
+  int clo[2] = {0, 0}, chi[2] = {0, 0}, cw = 0, ch = 0, pts = 0, rounds = 1;
+  std::set<Ver> need_sts;          // in-group versions still written to their SMEM ring
+  std::vector<std::vector<int>> phases;   // kernels between barriers
+  std::map<CanvasKey, Rect> krect; // shared loads and the rect of lanes that issue them
+  double lds_bytes = 0, sts_bytes = 0, tma_bytes = 0;   // per fast iteration per U planes
+};
+bool canvas_forward(const Program& p, const GroupLowering& L, int k, int x, const Off& d, int uu, int* prod, int* up);
+CanvasKey canvas_key(const Program& p, const GroupLowering& L, const CanvasPlan& c, int k, int x, const Off& d, int uu);
+Rect canvas_rect(const GroupLowering& L, const CanvasPlan& c, int k);
+CanvasPlan plan_canvas(const Program& p, const GroupLowering& L);
 
 // ---------------------------------------------------------------- codegen
 struct Codegen {

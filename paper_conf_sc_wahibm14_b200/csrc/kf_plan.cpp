@@ -9,6 +9,7 @@
 // The projection is the codeless upper bound of P:321 reduced to compulsory bytes over
 // peak bandwidth (Eq. 11's LD/ST counts).
 #include <algorithm>
+#include <cstdio>
 #include <climits>
 #include <cstring>
 
@@ -453,6 +454,14 @@ double model_time(const Program& p, const GroupLowering& L, const kf_target& t, 
   const double eff = std::min(1.0, warps / 32.0);
   const double t_comp = double(p.npts) * work / (2.5e13 * eff);
   const double t_mem = double(bytes) / (0.79 * t.hbm_bytes_per_s);
+  // shared-memory bandwidth (the canvas plan's loads, ring stores and TMA writes per tile plane) at
+  // 128 B/clk/SM on n_sm SMs at 1.9 GHz
+  const CanvasPlan cv = plan_canvas(p, L);
+  const double per_plane = (cv.lds_bytes + cv.sts_bytes + cv.tma_bytes) / std::max(1, L.zunroll);
+  const double t_smem = double(p.npts) / T * per_plane / (128.0 * t.n_sm * 1.9e9);
+  if (getenv("KF_DEBUG_MODEL"))
+    fprintf(stderr, "model: group of %zu kernels: mem %.3f ms, smem %.3f ms (lds %.0f sts %.0f tma %.0f B/plane, canvas %d), comp %.3f ms\n",
+            L.kernels.size(), t_mem * 1e3, t_smem * 1e3, cv.lds_bytes, cv.sts_bytes, cv.tma_bytes, int(cv.ok), t_comp * 1e3);
   return t_mem + t_comp - 0.5 * std::min(t_mem, t_comp) + 5e-6;
 }
 

@@ -1,0 +1,27 @@
+"""ncu driver: run `steps` steps of one weather plan (labels JSON, or hgga/hand) with one target.
+
+  ncu ... python tools/prof_plan.py '<plan>' '<target json>' [steps]
+"""
+import json, os, sys
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch
+import paper_conf_sc_wahibm14_b200 as kf
+from workloads import programs as P, data as D
+sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+from ab import HGGA
+
+desc = P.weather(n=(512, 512, 128))
+prog = kf.Program(desc)
+which = sys.argv[1]
+plan = {"hgga": HGGA, "hand": P.weather_hand_plan(desc)}.get(which) or json.loads(which)
+kw = {k: (tuple(v) if isinstance(v, list) else v) for k, v in json.loads(sys.argv[2] if len(sys.argv) > 2 else "{}").items()}
+steps = int(sys.argv[3]) if len(sys.argv) > 3 else 2
+ex = kf.Exec(prog, plan, kf.Target(**kw))
+ex.set_graph(False)
+dev = kf.device_arrays(prog, D.weather_inputs(desc, 3))
+sb = ex.scratch_bytes()
+scr = torch.empty(sb, dtype=torch.uint8, device="cuda") if sb else None
+ex.run(dev, scr, steps)
+torch.cuda.synchronize()
+print("done", [(ex.group_info(g).name.decode(), ex.group_info(g).threads, ex.group_info(g).regs, ex.group_info(g).smem_bytes)
+               for g in range(ex.info().n_groups)])
