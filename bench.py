@@ -38,7 +38,7 @@ def workload(name: str):
     from workloads import data, programs
     if name == "weather":
         desc = programs.weather(n=(512, 512, 128))
-        return desc, data.weather_inputs, dict(tile=(32, 8, 0)), "weather-44k31a-512x512x128-fp64 (BASELINE config 3)"
+        return desc, data.weather_inputs, dict(tile=(32, 8, 64)), "weather-44k31a-512x512x128-fp64 (BASELINE config 3)"
     if name == "weather_small":
         desc = programs.weather(n=(128, 128, 64))
         return desc, data.weather_inputs, dict(tile=(32, 16, 0)), "weather-44k31a-128x128x64-fp64"
@@ -55,6 +55,64 @@ def workload(name: str):
         desc = programs.stress(m=2, n=(768, 768, 768))
         return desc, None, dict(tile=(32, 8, 0), max_halo=16), "stress-2fields-L25xL25-768^3-fp64 (config 5)"
     raise SystemExit(f"unknown workload {name}")
+
+
+def plan_candidates(prog, target):
+    """Candidate plans for measured selection: the paper's search (HGGA) on the projected
+    time with three seeds and on compulsory bytes, greedy merging on projected time, and (weather)
+    the App. A.4 hand plan.  Deduplicated by canonical labelling."""
+    import paper_conf_sc_wahibm14_b200 as kf
+    out, seen = [], set()
+
+    def add(plan, kind):
+        canon, m = [], {}
+        for g in plan:
+            canon.append(m.setdefault(g, len(m)))
+        if tuple(canon) not in seen:
+            seen.add(tuple(canon))
+            out.append((canon, kind))
+    if prog.nk <= 10:
+        add(prog.search(kf.SEARCH_BRUTE_TIME, target)[0], "brute-force on projected time")
+        add(prog.search(kf.SEARCH_BRUTE, target)[0], "brute-force on compulsory bytes")
+    else:
+        for seed in (1, 2, 3):
+            add(prog.search(kf.SEARCH_HGGA, target, seed=seed)[0], f"HGGA (seed {seed}) on the resource-aware projected time")
+        add(prog.search(kf.SEARCH_HGGA_BYTES, target, seed=1)[0], "HGGA (seed 1) on compulsory bytes")
+        add(prog.search(kf.SEARCH_GREEDY_TIME, target)[0], "greedy merging on projected time")
+    if prog.desc.name == "weather":
+        from workloads.programs import weather_hand_plan
+        add(weather_hand_plan(prog.desc), "hand plan (App. A.4)")
+    return out
+
+
+def select_plan(prog, target, dev, steps=5):
+    """Measured selection among plan_candidates(): every candidate is compiled with the default
+    launch configuration and timed (CUDA events, `steps` steps after 2 warm-up steps); the
+    fastest is kept.  The projection ranks plans inside the search; the measurement decides
+    between the few it proposes."""
+    import torch
+    import paper_conf_sc_wahibm14_b200 as kf
+    res = []
+    for plan, kind in plan_candidates(prog, target):
+        try:
+            ex = kf.Exec(prog, plan, target)
+        except Exception as e:   # an illegal candidate for this target: skip it
+            res.append((float("inf"), plan, kind + f" (failed: {str(e)[:80]})"))
+            continue
+        sb = ex.scratch_bytes()
+        scr = torch.empty(sb, dtype=torch.uint8, device="cuda") if sb else None
+        ex.run(dev, scr, 2)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        ex.run(dev, scr, steps)
+        e1.record()
+        torch.cuda.synchronize()
+        res.append((e0.elapsed_time(e1) / steps, plan, kind))
+        del ex, scr
+    best = min(res, key=lambda r: r[0])
+    return best[1], best[2] + " (fastest of the measured candidates)", [
+        {"plan": kind, "ms_per_step": round(ms, 4), "groups": len(set(plan))} for ms, plan, kind in res]
 
 
 def choose_plan(prog, target, which: str):
@@ -299,7 +357,7 @@ def run_kf(args):
         tkw["threads"] = args.threads
     target = kf.Target(**tkw)
     prog = kf.Program(desc)          # the per-GPU sub-domain program (weak scaling)
-    plan, plan_kind = choose_plan(prog, target, args.plan)
+    plan, plan_kind = (None, None) if args.plan == "select" else choose_plan(prog, target, args.plan)
     dist_info = None
     if world > 1:
         px, py = grid_for(world)
@@ -320,6 +378,14 @@ def run_kf(args):
         del inputs
     stream = torch.cuda.current_stream()
     t0 = time.time()
+    candidates = None
+    if plan is None:   # measured plan selection (rank 0 decides, every rank runs the same plan)
+        if rank == 0:
+            plan, plan_kind, candidates = select_plan(prog, target, dev)
+        if world > 1:
+            obj = [(plan, plan_kind, candidates)]
+            torch.distributed.broadcast_object_list(obj, 0)
+            plan, plan_kind, candidates = obj[0]
     tuned, gtargets = None, None
     if args.tuned:   # fixed per-group configs (e.g. for an ncu run of exactly the timed configuration)
         tuned = json.loads(args.tuned)
@@ -418,7 +484,8 @@ def run_kf(args):
                    "parallelism": (f"xy domain decomposition {grid_for(world)[0]}x{grid_for(world)[1]}, NCCL halo "
                                    f"exchange, weak (512x512x128 per GPU)") if world > 1 else "1 GPU",
                    "graph": world == 1, "jit_s": round(jit_s, 2),
-                   "per_group_launch_config": tuned if tuned else "uniform"},
+                   "per_group_launch_config": tuned if tuned else "uniform",
+                   "plan_candidates": candidates},
         "hbm_gbs_compulsory": achieved_step,
         "frac_of_measured_copy": achieved_step / hbm_peak,
         "frac_of_nominal_8TBs": achieved_step / 8000.0,
@@ -492,7 +559,8 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="kf", choices=["kf", "reference"])
     ap.add_argument("--workload", default="weather")
-    ap.add_argument("--plan", default="best", choices=["best", "unfused", "hand"])
+    ap.add_argument("--plan", default="select", choices=["select", "best", "unfused", "hand"],
+                    help="select: measured choice among the searches' candidates; best: HGGA/brute on projected time")
     ap.add_argument("--relax-all", type=int, default=0, help="weather: rename every written array (KF_PROG_RELAX_ALL)")
     ap.add_argument("--tile", default=None)
     ap.add_argument("--stages", type=int, default=None)
