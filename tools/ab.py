@@ -56,7 +56,8 @@ def main():
         torch.cuda.synchronize()
         gms, _ = ex.group_times()
         gi = [ex.group_info(g) for g in range(ex.info().n_groups)]
-        print(json.dumps({"variant": v, "ms_per_step": round(ms, 4),
+        jit = [prog.jit_check(plan, g, kf.Target(**kw))[0] for g in range(len(gi))] if os.environ.get("AB_JIT") else None
+        print(json.dumps({"variant": v, "ms_per_step": round(ms, 4), "jit_regs": jit,
                           "groups": [(g.name.decode(), round(t / steps, 4), g.regs, g.smem_bytes) for g, t in zip(gi, gms)]}),
               flush=True)
         del ex, scr
