@@ -169,10 +169,10 @@ typedef struct {
                                     unrolled so every SMEM slot is a compile-time constant    */
   int32_t ghostwrite;            /* 1: stores also write periodic x/y ghost copies, so the step
                                     needs no ghost-fill kernels (single-domain runs)          */
-  int32_t minblocks;             /* __launch_bounds__ minimum CTAs per SM of the group kernels:
-                                    0 = as many as shared memory allows (registers then never cut
-                                    occupancy below it; recompiled with 1 if ptxas would spill),
-                                    -1 = no bound, n >= 1 = n                                  */
+  int32_t minblocks;             /* register cap of the group kernels (__maxnreg__): keep this
+                                    many CTAs per SM resident -- 0 = as many as shared memory
+                                    allows, n >= 1 = n; never above R_est (V8); dropped if ptxas
+                                    would spill.  -1 = no cap                                   */
   int32_t pad;
 } kf_target;
 /* Fills the B200 defaults: 8.0e12, 232448, 255, 148, {64,4,0}, 2, 256, 16, 0, 1, {1,1}, 0, 0, 0. */

@@ -128,9 +128,9 @@ static std::shared_ptr<Compiled> compile_cached(const std::string& src, const st
     if (it != g_cubin_cache.end()) return it->second;
   }
   auto c = std::make_shared<Compiled>(nvrtc_compile(src, name));
-  // the occupancy bound of __launch_bounds__ (KF_MINB) must not cost local-memory spills
-  if (c->spill > 0 && src.find("#define KF_MINB") != std::string::npos)
-    c = std::make_shared<Compiled>(nvrtc_compile("#define KF_MINB 1\n" + src, name));
+  // the register cap (__maxnreg__, occupancy) must not cost local-memory spills
+  if (c->spill > 0 && src.find("__maxnreg__") != std::string::npos)
+    c = std::make_shared<Compiled>(nvrtc_compile("#define KF_NO_MAXNREG 1\n" + src, name));
   std::lock_guard<std::mutex> lk(g_cache_mu);
   g_cubin_cache[src] = c;
   return c;
