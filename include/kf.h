@@ -173,9 +173,12 @@ typedef struct {
                                     many CTAs per SM resident -- 0 = as many as shared memory
                                     allows, n >= 1 = n; never above R_est (V8); dropped if ptxas
                                     would spill.  -1 = no cap                                   */
-  int32_t pad;
+  int32_t skew;                  /* 1: a kernel reading an in-group version at a nonzero xy offset
+                                    runs U more planes behind its producer (delay skew, R20c), so
+                                    it reads planes the previous iteration's barrier published and
+                                    fast iterations need no barrier between kernels             */
 } kf_target;
-/* Fills the B200 defaults: 8.0e12, 232448, 255, 148, {64,4,0}, 2, 256, 16, 0, 1, {1,1}, 0, 0, 0. */
+/* Fills the B200 defaults: 8.0e12, 232448, 255, 148, {64,4,0}, 2, 256, 16, 0, 1, {1,1}, 0, 0, 0, 0. */
 kf_status kf_target_b200(kf_target* out);
 
 /* ------------------------------------------------------------------ legality (Eq. 1.1-1.7) */

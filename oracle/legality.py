@@ -44,6 +44,7 @@ class Target:
     zunroll: int = 1                # planes per stream iteration U (ring depth grows with U, R20)
     pblock: Tuple[int, int] = (1, 1)  # points per thread in x, y (register blocking)
     ringunroll: int = 0             # 1: ring depths rounded up to powers of two (R20b)
+    skew: int = 0                   # 1: reads at a nonzero xy offset of in-group versions lag U more planes (R20c)
 
 
 # ---------------------------------------------------------------- plans
@@ -177,7 +178,8 @@ def schedule(prog: Program, grp: List[int], target: Target):
     with their boxes, ring slots and bytes.  The definition the CUDA kernel must fit (R20)."""
     ext, pts = extended_regions(prog, grp)
     alive = [k for k in grp if ext[k] is not None]
-    # delays: a consumer runs D_p + dz planes behind the producer of what it reads
+    # delays: a consumer runs D_p + dz planes behind the producer of what it reads; with the delay
+    # skew (R20c) a read at a nonzero xy offset runs U planes further behind
     D: Dict[int, int] = {}
     for k in alive:
         dk = 0
@@ -185,7 +187,9 @@ def schedule(prog: Program, grp: List[int], target: Target):
             v = G.version_read(prog, k, x)
             if v >= 1 and G.writer_of(prog, x, v) in alive:
                 p = G.writer_of(prog, x, v)
-                dk = max(dk, D[p] + max(d[2] for d in offs))
+                for d in offs:
+                    lag = target.zunroll if (target.skew and (d[0] != 0 or d[1] != 0)) else 0
+                    dk = max(dk, D[p] + d[2] + lag)
         D[k] = dk
     es = prog.es
     TX, TY = target.tile[0], target.tile[1]

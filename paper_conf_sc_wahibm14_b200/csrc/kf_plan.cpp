@@ -124,7 +124,9 @@ GroupLowering lower_group(const Program& p, const std::vector<int>& g, const kf_
   std::vector<int> alive;
   for (int k : g)
     if (L.ext[k].alive) alive.push_back(k);
-  // ---- z delays: a consumer runs behind its in-group producers by their dz reach
+  // ---- z delays: a consumer runs behind its in-group producers by their dz reach; with the delay
+  // skew (R20c) reads at a nonzero xy offset stay U planes further behind, so they only touch
+  // planes written in earlier iterations (published by the end-of-iteration barrier)
   for (int k : alive) {
     int dk = 0;
     for (auto& [x, offs] : p.kernels[k].reads) {
@@ -132,9 +134,10 @@ GroupLowering lower_group(const Program& p, const std::vector<int>& g, const kf_
       if (v < 1) continue;
       int pr = p.writer_of(x, v);
       if (!in_group(g, pr) || !L.ext[pr].alive) continue;
-      int mz = INT_MIN;
-      for (auto& d : offs) mz = std::max(mz, d[2]);
-      dk = std::max(dk, L.delay[pr] + mz);
+      for (auto& d : offs) {
+        const bool xy = d[0] != 0 || d[1] != 0;
+        dk = std::max(dk, L.delay[pr] + d[2] + (t.skew && xy ? t.zunroll : 0));
+      }
     }
     L.delay[k] = dk;
   }
@@ -477,6 +480,7 @@ void check_target(const kf_target* t) {
   if (t->ringunroll < 0 || t->ringunroll > 1) fail(KF_E_ARG, "ringunroll must be 0 or 1");
   if (t->ghostwrite < 0 || t->ghostwrite > 1) fail(KF_E_ARG, "ghostwrite must be 0 or 1");
   if (t->minblocks < -1 || t->minblocks > 32) fail(KF_E_ARG, "minblocks must be in [-1, 32]");
+  if (t->skew < 0 || t->skew > 1) fail(KF_E_ARG, "skew must be 0 or 1");
   if (t->pblock[0] < 1 || t->pblock[0] > 4 || t->pblock[1] < 1 || t->pblock[1] > 4)
     fail(KF_E_ARG, "pblock must be in [1, 4] x [1, 4]");
   if (t->threads < 32 || t->threads > 1024 || t->threads % 32) fail(KF_E_ARG, "threads must be a multiple of 32 in [32,1024]");

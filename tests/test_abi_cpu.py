@@ -125,11 +125,13 @@ def test_resource_limits_V7_V8():
         check_program(desc, target=(L.Target(zunroll=zu, tile=(16, 8, 0)), kf.Target(zunroll=zu, tile=(16, 8, 0))))
     for kw in (dict(pblock=(2, 2), zunroll=2, threads=128, tile=(32, 8, 0)), dict(pblock=(1, 3), threads=64, tile=(16, 16, 0)),
                dict(pblock=(4, 1), threads=32, tile=(64, 4, 0)), dict(ringunroll=1, zunroll=2, tile=(32, 8, 0)),
-               dict(ringunroll=1, tile=(16, 16, 0), stages=3)):
+               dict(ringunroll=1, tile=(16, 16, 0), stages=3), dict(skew=1, tile=(32, 8, 0)),
+               dict(skew=1, zunroll=2, tile=(16, 8, 0))):
         check_program(P.fig3(), target=(L.Target(**kw), kf.Target(**kw)))
     tk = kf.Target(regs_per_thread_max=40, zunroll=2)
     to = L.Target(regs_per_thread_max=40, zunroll=2)
     check_program(desc, target=(to, tk))
+    check_program(desc, target=(L.Target(skew=1), kf.Target(skew=1)))
 
 
 def test_weather_program_abi_and_greedy():

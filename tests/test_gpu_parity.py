@@ -201,3 +201,48 @@ def test_stress_config5_radius4_plans(tile):
         assert compare(desc, got, ref) == [], plan
         n += 1
     assert n == prog.count_legal(tgt) >= 4
+
+
+@pytest.mark.parametrize("seed", range(8))
+def test_canvas_paths_random_programs(seed, monkeypatch):
+    """Canvas fast iterations (one canvas point per thread: register forwarding, cross-kernel load
+    CSE) under every codegen knob: delay skew, z-queue carries (KF_CQ), register cap, z-unroll."""
+    rng = np.random.default_rng(3000 + seed)
+    bc = tuple(int(x) for x in rng.integers(0, 2, size=3))
+    flags = [0, PROG_RELAX_EXPANDABLE, PROG_RELAX_ALL][seed % 3]
+    dtype = DT_F64 if seed % 2 else DT_F32
+    n = tuple(int(x) for x in rng.integers(12, 40, size=3))
+    desc = P.random_program(4000 + seed, nk=6, na=4, n=n, dtype=dtype, bc=bc, flags=flags, max_r=1 + seed % 2)
+    inputs = D.uniform(desc, seed)
+    nsteps = 1 + seed % 2
+    ref = interp.run(desc, inputs, nsteps)
+    legal = En.legal_plans(desc)
+    # the plans with the largest groups exercise forwarding the most
+    pick = sorted(legal, key=lambda p: len(set(p)))[:3]
+    if seed % 2:
+        monkeypatch.setenv("KF_CQ", "1")
+    tile = [(16, 8, 0), (8, 8, 7), (32, 4, 0), (16, 4, 9)][seed % 4]
+    for plan in pick:
+        for skew, mb, zu in ((0, 0, 1), (1, -1, 1), (seed % 2, 0, 2)):
+            got, _ = run_kf(desc, plan, inputs, nsteps, kf.Target(tile=tile, skew=skew, minblocks=mb, zunroll=zu))
+            assert compare(desc, got, ref) == [], (plan, tile, skew, mb, zu)
+
+
+@pytest.mark.parametrize("cq", [0, 1])
+def test_canvas_weather_knobs(cq, monkeypatch):
+    """Weather program (config 3 shape, small grid): the bench's plan family with the canvas knobs."""
+    if cq:
+        monkeypatch.setenv("KF_CQ", "1")
+    desc = P.weather(n=(64, 48, 12))
+    inputs = D.inputs_for(desc, 4)
+    ref = interp.run(desc, inputs, 2)
+    prog = kf.Program(desc)
+    tgt = kf.Target(tile=(32, 8, 0))
+    plans = [prog.search(kf.SEARCH_HGGA, tgt, seed=s)[0] for s in (1, 2)]
+    for plan in plans:
+        for kw in (dict(), dict(skew=1), dict(minblocks=-1, ringunroll=1), dict(tile=(32, 8, 5))):
+            t = kf.Target(**dict(dict(tile=(32, 8, 0)), **kw))
+            if kw and prog.validate(plan, t)[0] != 0:   # e.g. V7: skew / ring unrolling need more SMEM
+                continue
+            got, _ = run_kf(desc, plan, inputs, 2, t)
+            assert compare(desc, got, ref) == [], (plan, kw)
