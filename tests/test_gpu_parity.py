@@ -246,3 +246,17 @@ def test_canvas_weather_knobs(cq, monkeypatch):
                 continue
             got, _ = run_kf(desc, plan, inputs, 2, t)
             assert compare(desc, got, ref) == [], (plan, kw)
+
+
+@pytest.mark.parametrize("nk,load", [(30, 4), (40, 8), (24, 12)])
+def test_suite_sweep_programs_parity(nk, load):
+    """NEXT-3 test-suite programs (Table V thread loads 4/8/12): the HGGA plans vs the oracle."""
+    desc = P.gen_suite(n_kernels=nk, n_arrays=2 * nk, seed=1, n=(40, 32, 12), load=load, max_tries=2000)
+    inputs = D.uniform(desc, 7)
+    ref = interp.run(desc, inputs, 2)
+    prog = kf.Program(desc)
+    tgt = kf.Target(tile=(32, 8, 0))
+    for method in (kf.SEARCH_HGGA, kf.SEARCH_HGGA_BYTES):
+        plan, _ = prog.search(method, tgt, seed=1)
+        got, _ = run_kf(desc, plan, inputs, 2, tgt)
+        assert compare(desc, got, ref) == [], (method, plan)

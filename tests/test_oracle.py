@@ -467,3 +467,18 @@ def test_paper_eq8_worked_example_golden():
     assert r["b_sh"] == gold["printed"]["b_sh"]
     assert r["p_membound_gflops"] == 688 * 14 * 202 / (8 * 128 * 64) == gold["derived_from_printed_formula"]["p_membound_gflops"]
     assert round(100 * r["p_membound_gflops"] / gold["printed"]["roofline_gflops"], 2) == gold["derived_from_printed_formula"]["percent"]
+
+
+def test_suite_generator_thread_load_and_sharing_sets():
+    """NEXT-3 generator: the average thread load (distinct offsets per kernel-array read, R10) follows
+    Table V's parameter and every sharing set stays within 2..8 kernels."""
+    from oracle import graph as Gr
+    for nk, load in ((30, 4), (60, 8), (100, 12)):
+        d = P.gen_suite(n_kernels=nk, n_arrays=2 * nk, seed=1, n=(8, 8, 4), load=load, max_tries=2000)
+        loads = [len(offs) for k in range(nk) for offs in Gr.reads(d, k).values()]
+        assert abs(sum(loads) / len(loads) - load) < 1.0, (nk, load, sum(loads) / len(loads))
+        users = {}
+        for k in range(nk):
+            for x in set(Gr.reads(d, k)) | set(Gr.writes(d, k)):
+                users.setdefault(x, set()).add(k)
+        assert all(len(u) <= 8 for u in users.values())
