@@ -358,13 +358,15 @@ def run_kf(args):
     target = kf.Target(**tkw)
     prog = kf.Program(desc)          # the per-GPU sub-domain program (weak scaling)
     plan, plan_kind = (None, None) if args.plan == "select" else choose_plan(prog, target, args.plan)
-    dist_info = None
-    if world > 1:
+    def new_dist_info():
+        """A fresh NCCL unique id (broadcast from rank 0) for every communicator kf.Dist creates."""
+        if world == 1:
+            return None
         px, py = grid_for(world)
         nid = kf.dist_unique_id() if rank == 0 else bytes(128)
         t = torch.tensor(list(nid), dtype=torch.uint8, device="cuda")
         torch.distributed.broadcast(t, 0)
-        dist_info = (px, py, rank, world, bytes(t.cpu().tolist()))
+        return (px, py, rank, world, bytes(t.cpu().tolist()))
     # synthetic inputs of the paper-shaped workload (seed 3 + rank: each rank owns its sub-domain)
     if gen is None:
         # large uniform workloads: U[-1,1) generated on the device (seeded torch generator)
@@ -402,7 +404,7 @@ def run_kf(args):
             gtargets = [kf.Target(**dict(tkw, tile=tuple(c[0]), stages=c[1], zunroll=c[2], ringunroll=c[3],
                                             minblocks=c[4] if len(c) > 4 else 0))
                         for c in tuned]
-    rn = Runner(prog, plan, target, gtargets, dist_info)
+    rn = Runner(prog, plan, target, gtargets, new_dist_info())
     jit_s = time.time() - t0
     info = rn.ex.info()
     npts = desc.npts
@@ -416,7 +418,7 @@ def run_kf(args):
     # unfused plan on the same inputs: speedup vs unfused
     unf = None
     if not args.no_unfused and args.plan != "unfused":
-        rn_u = Runner(prog, list(range(prog.nk)), target, None, dist_info)
+        rn_u = Runner(prog, list(range(prog.nk)), target, None, new_dist_info())
         ms_u, _ = time_runner(rn_u, dev, args.steps, args.warmup, stream)
         ms_u = max_over_ranks(ms_u)
         unf = {"ms_per_step": ms_u / args.steps, "bytes_per_step": rn_u.ex.info().compulsory_bytes_per_step}
