@@ -131,57 +131,81 @@ def choose_plan(prog, target, which: str):
 
 # ---------------------------------------------------------------- clocks
 class ClockSampler:
-    FIELDS = "clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown," \
-             "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown," \
-             "clocks_event_reasons.sw_power_cap"
+    """SM clock and clock-event reasons sampled through NVML every 5 ms DURING the timed region
+    (a thread started before it, stopped after it); only samples taken while the region ran count."""
+    REASONS = (("hw_slowdown", "nvmlClocksEventReasonHwSlowdown"),
+               ("hw_thermal_slowdown", "nvmlClocksEventReasonHwThermalSlowdown"),
+               ("sw_thermal_slowdown", "nvmlClocksEventReasonSwThermalSlowdown"),
+               ("sw_power_cap", "nvmlClocksEventReasonSwPowerCap"),
+               ("hw_power_brake", "nvmlClocksEventReasonHwPowerBrakeSlowdown"))
 
     def __init__(self, index: int):
         self.index = index
-        self.proc = None
-        self.lines = []
+        self.samples = []
+        self.err = None
+        self.h = None
+        self.stop = threading.Event()
+        self.t0 = self.t1 = None
 
     def __enter__(self):
         try:
-            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
-                                          "--format=csv,noheader,nounits", "-lms", "50"],
-                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
-            self.t = threading.Thread(target=self._read, daemon=True)
-            self.t.start()
-        except Exception:
-            self.proc = None
+            import pynvml
+            import torch
+            self.nv = pynvml
+            pynvml.nvmlInit()
+            try:
+                uuid = str(torch.cuda.get_device_properties(self.index).uuid)
+                self.h = pynvml.nvmlDeviceGetHandleByUUID(uuid if uuid.startswith("GPU-") else "GPU-" + uuid)
+            except Exception:
+                self.h = pynvml.nvmlDeviceGetHandleByIndex(self.index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.th = threading.Thread(target=self._loop, daemon=True)
+            self.th.start()
+        except Exception as e:  # no NVML: reported as unavailable, never guessed
+            self.err = f"{type(e).__name__}: {e}"
+            self.h = None
         return self
 
-    def _read(self):  # noqa: D401
-        for line in self.proc.stdout:
-            self.lines.append(line.strip())
+    def mark_start(self):
+        self.t0 = time.perf_counter()
+
+    def mark_end(self):
+        self.t1 = time.perf_counter()
+
+    def _loop(self):
+        nv = self.nv
+        while not self.stop.is_set():
+            try:
+                t = time.perf_counter()
+                sm = nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM)
+                rs = nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                self.samples.append((t, sm, rs))
+            except Exception as e:
+                self.err = f"{type(e).__name__}: {e}"
+                return
+            time.sleep(0.005)
 
     def __exit__(self, *a):
-        if self.proc:
-            self.proc.terminate()
-            try:
-                self.proc.wait(timeout=5)
-            except Exception:
-                self.proc.kill()
+        self.stop.set()
+        if self.h is not None:
+            self.th.join(timeout=2)
 
     def summary(self):
-        sm, mx, reasons = [], None, set()
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for ln in self.lines:
-            parts = [p.strip() for p in ln.split(",")]
-            if len(parts) < 7:
-                continue
-            try:
-                sm.append(float(parts[0]))
-                mx = float(parts[1])
-            except ValueError:
-                continue
-            for nm, v in zip(names, parts[3:7]):
-                if v.lower() in ("active", "1"):
+        if self.h is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"], "error": self.err}
+        t0 = self.t0 if self.t0 is not None else float("-inf")
+        t1 = self.t1 if self.t1 is not None else float("inf")
+        win = [s for s in self.samples if t0 <= s[0] <= t1]
+        if not win:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": ["no sample in the timed region"]}
+        sm = sorted(s[1] for s in win)
+        reasons = set()
+        for _, _, rs in win:
+            for nm, attr in self.REASONS:
+                if rs & getattr(self.nv, attr, 0):
                     reasons.add(nm)
-        if not sm:
-            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"]}
-        sm.sort()
-        return {"sm_mhz": sm[len(sm) // 2], "sm_max_mhz": mx, "reasons": sorted(reasons), "samples": len(sm)}
+        return {"sm_mhz": sm[len(sm) // 2], "sm_max_mhz": self.max_mhz, "reasons": sorted(reasons),
+                "samples": len(win), "source": "NVML, 5 ms, inside the timed region"}
 
 
 def measured_peaks():
@@ -305,7 +329,7 @@ class Runner:
             self.dist.run([dev], [self.scratch], nsteps, stream=stream)
 
 
-def time_runner(rn, dev, steps, warmup, stream, profile=False):
+def time_runner(rn, dev, steps, warmup, stream, profile=False, clk=None):
     import torch
     rn.run(dev, warmup, stream)
     torch.cuda.synchronize()
@@ -316,10 +340,14 @@ def time_runner(rn, dev, steps, warmup, stream, profile=False):
     torch.cuda.synchronize()
     e0 = torch.cuda.Event(enable_timing=True)
     e1 = torch.cuda.Event(enable_timing=True)
+    if clk is not None:
+        clk.mark_start()
     e0.record(stream)
     rn.run(dev, steps, stream)
     e1.record(stream)
     torch.cuda.synchronize()
+    if clk is not None:
+        clk.mark_end()
     ms = e0.elapsed_time(e1)
     gt = None
     if profile:
@@ -410,7 +438,7 @@ def run_kf(args):
     npts = desc.npts
 
     with ClockSampler(local) as clk:
-        ms, _ = time_runner(rn, dev, args.steps, args.warmup, stream)
+        ms, _ = time_runner(rn, dev, args.steps, args.warmup, stream, clk=clk)
     ms = max_over_ranks(ms)
     clocks = clk.summary()
     # per-group device times over a second timed region (events on the launch stream)
