@@ -177,8 +177,12 @@ typedef struct {
                                     runs U more planes behind its producer (delay skew, R20c), so
                                     it reads planes the previous iteration's barrier published and
                                     fast iterations need no barrier between kernels             */
+  int32_t canvas_ld;             /* fast-iteration shared loads: 1 = unpredicated wherever every
+                                    address they can form lies in the rings' SMEM (fewer
+                                    instructions; lanes outside the readers' regions load values
+                                    nobody stores), 0 = predicated on the readers' regions      */
 } kf_target;
-/* Fills the B200 defaults: 8.0e12, 232448, 255, 148, {64,4,0}, 2, 256, 16, 0, 1, {1,1}, 0, 0, 0, 0. */
+/* Fills the B200 defaults: 8.0e12, 232448, 255, 148, {64,4,0}, 2, 256, 16, 0, 1, {1,1}, 0, 0, 0, 0, 1. */
 kf_status kf_target_b200(kf_target* out);
 
 /* ------------------------------------------------------------------ legality (Eq. 1.1-1.7) */

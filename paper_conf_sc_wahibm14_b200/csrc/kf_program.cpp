@@ -348,6 +348,7 @@ kf_status kf_target_b200(kf_target* out) {
     t.ghostwrite = 0;   // measured slower than the fill kernels on B200 (tools/sweep.py, round 1)
     t.minblocks = 0;
     t.skew = 0;
+    t.canvas_ld = 1;
     *out = t;
   });
 }

@@ -206,7 +206,8 @@ def test_stress_config5_radius4_plans(tile):
 @pytest.mark.parametrize("seed", range(8))
 def test_canvas_paths_random_programs(seed, monkeypatch):
     """Canvas fast iterations (one canvas point per thread: register forwarding, cross-kernel load
-    CSE) under every codegen knob: delay skew, z-queue carries (KF_CQ), register cap, z-unroll."""
+    CSE) under every codegen knob: delay skew, z-queue carries (KF_CQ), register cap, z-unroll,
+    unpredicated / predicated shared loads (canvas_ld)."""
     rng = np.random.default_rng(3000 + seed)
     bc = tuple(int(x) for x in rng.integers(0, 2, size=3))
     flags = [0, PROG_RELAX_EXPANDABLE, PROG_RELAX_ALL][seed % 3]
@@ -223,9 +224,9 @@ def test_canvas_paths_random_programs(seed, monkeypatch):
         monkeypatch.setenv("KF_CQ", "1")
     tile = [(16, 8, 0), (8, 8, 7), (32, 4, 0), (16, 4, 9)][seed % 4]
     for plan in pick:
-        for skew, mb, zu in ((0, 0, 1), (1, -1, 1), (seed % 2, 0, 2)):
-            got, _ = run_kf(desc, plan, inputs, nsteps, kf.Target(tile=tile, skew=skew, minblocks=mb, zunroll=zu))
-            assert compare(desc, got, ref) == [], (plan, tile, skew, mb, zu)
+        for skew, mb, zu, cl in ((0, 0, 1, 1), (0, 0, 1, 0), (1, -1, 1, 1), (seed % 2, 0, 2, seed % 2)):
+            got, _ = run_kf(desc, plan, inputs, nsteps, kf.Target(tile=tile, skew=skew, minblocks=mb, zunroll=zu, canvas_ld=cl))
+            assert compare(desc, got, ref) == [], (plan, tile, skew, mb, zu, cl)
 
 
 @pytest.mark.parametrize("cq", [0, 1])
@@ -240,7 +241,7 @@ def test_canvas_weather_knobs(cq, monkeypatch):
     tgt = kf.Target(tile=(32, 8, 0))
     plans = [prog.search(kf.SEARCH_HGGA, tgt, seed=s)[0] for s in (1, 2)]
     for plan in plans:
-        for kw in (dict(), dict(skew=1), dict(minblocks=-1, ringunroll=1), dict(tile=(32, 8, 5))):
+        for kw in (dict(), dict(canvas_ld=0), dict(skew=1), dict(minblocks=-1, ringunroll=1), dict(tile=(32, 8, 5))):
             t = kf.Target(**dict(dict(tile=(32, 8, 0)), **kw))
             if kw and prog.validate(plan, t)[0] != 0:   # e.g. V7: skew / ring unrolling need more SMEM
                 continue
