@@ -123,6 +123,8 @@ def choose_plan(prog, target, which: str):
     if which == "hand":
         from workloads.programs import weather_hand_plan
         return weather_hand_plan(prog.desc), "hand plan (App. A.4)"
+    if which.startswith("["):   # explicit labels, e.g. config.plan_labels of an earlier run
+        return [int(v) for v in json.loads(which)], "given labels"
     method = kf.SEARCH_BRUTE_TIME if n <= 10 else kf.SEARCH_HGGA
     plan, _ = prog.search(method, target, seed=1)
     return plan, ("brute-force on projected time" if method == kf.SEARCH_BRUTE_TIME
@@ -594,8 +596,9 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="kf", choices=["kf", "reference"])
     ap.add_argument("--workload", default="weather")
-    ap.add_argument("--plan", default="select", choices=["select", "best", "unfused", "hand"],
-                    help="select: measured choice among the searches' candidates; best: HGGA/brute on projected time")
+    ap.add_argument("--plan", default="select",
+                    help="select: measured choice among the searches' candidates; best: HGGA/brute on projected "
+                         "time; unfused; hand; or a JSON label list (config.plan_labels of an earlier run)")
     ap.add_argument("--relax-all", type=int, default=0, help="weather: rename every written array (KF_PROG_RELAX_ALL)")
     ap.add_argument("--tile", default=None)
     ap.add_argument("--stages", type=int, default=None)

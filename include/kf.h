@@ -305,7 +305,7 @@ kf_status kf_run_host(kf_exec* ex, void* const* host_arrays, int64_t nsteps, con
 typedef struct {
   int32_t n_groups;             /* fused kernels launched per step                        */
   int32_t launches_per_step;    /* group kernels + ghost fills                            */
-  int32_t fills_per_step;
+  int32_t fills_per_step;       /* ghost-fill kernel launches per step (consecutive fills batched) */
   int32_t period;               /* steps per replay period (2 with renamed step-live)     */
   uint64_t compulsory_bytes_per_step;
 } kf_exec_info;

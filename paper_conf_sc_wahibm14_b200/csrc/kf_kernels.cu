@@ -60,6 +60,44 @@ __global__ void fill_z(T* __restrict__ base, Geom g) {
   }
 }
 
+// Periodic x and y ghosts of several buffers in one launch (blockIdx.y = buffer): every ghost
+// cell takes the interior cell its coordinates wrap to on the periodic axes (a frozen axis keeps
+// its coordinate), which is what fill_x followed by fill_y produces, corners included, without
+// the ordering between the two passes.  Pieces: the x-ghost columns of every padded row (if x
+// is periodic) and the y-ghost rows over the x range not already covered (if y is periodic).
+struct FillList { void* base[kMaxFillBufs]; };
+
+template <typename T>
+__global__ void fill_xy_multi(FillList L, Geom g, int px, int py) {
+  T* base = (T*)L.base[blockIdx.y];
+  const int NZ = g.nz + 2 * g.gz, NYp = g.ny + 2 * g.gy;
+  const long long nxs = px ? 2LL * g.gx * NYp * NZ : 0;                  // x-ghost columns
+  const int x_lo = px ? 0 : -g.gx, x_w = px ? g.nx : g.nx + 2 * g.gx;    // y rows: x range not in nxs
+  const long long nys = py ? (long long)x_w * 2 * g.gy * NZ : 0;
+  for (long long idx = blockIdx.x * (long long)blockDim.x + threadIdx.x; idx < nxs + nys;
+       idx += (long long)gridDim.x * blockDim.x) {
+    int i, j, k;
+    if (idx < nxs) {
+      const int e = int(idx % (2 * g.gx));
+      const long long r = idx / (2 * g.gx);
+      j = int(r % NYp) - g.gy;
+      k = int(r / NYp) - g.gz;
+      i = e < g.gx ? -1 - e : g.nx + (e - g.gx);
+    } else {
+      const long long q = idx - nxs;
+      i = x_lo + int(q % x_w);
+      const long long r = q / x_w;
+      const int e = int(r % (2 * g.gy));
+      k = int(r / (2 * g.gy)) - g.gz;
+      j = e < g.gy ? -1 - e : g.ny + (e - g.gy);
+    }
+    const int si = (px && (i < 0 || i >= g.nx)) ? (i < 0 ? i + g.nx : i - g.nx) : i;
+    const int sj = (py && (j < 0 || j >= g.ny)) ? (j < 0 ? j + g.ny : j - g.ny) : j;
+    const long long o = (long long)(k + g.gz) * g.plane + g.xoff;
+    base[o + (long long)(j + g.gy) * g.pitch + i] = base[o + (long long)(sj + g.gy) * g.pitch + si];
+  }
+}
+
 // Copy every element that is not interior (ghost shell and padding) from src to dst:
 // renamed copies of an array share its frozen ghost values (R9).
 template <typename T>
@@ -114,6 +152,24 @@ cudaError_t launch_fill(int axis, void* base, int es, const Geom& g, cudaStream_
     if (axis == 0) fill_x<double><<<nb, 256, 0, s>>>((double*)base, g);
     else if (axis == 1) fill_y<double><<<nb, 256, 0, s>>>((double*)base, g);
     else fill_z<double><<<nb, 256, 0, s>>>((double*)base, g);
+  }
+  return cudaGetLastError();
+}
+
+cudaError_t launch_fill_xy_multi(void* const* bufs, int n, int px, int py, int es, const Geom& g, cudaStream_t s) {
+  if (!px && !py) return cudaSuccess;
+  const long long per = (px ? 2LL * g.gx * (g.ny + 2 * g.gy) : 0) * (g.nz + 2 * g.gz) +
+                        (py ? (long long)(px ? g.nx : g.nx + 2 * g.gx) * 2 * g.gy * (g.nz + 2 * g.gz) : 0);
+  if (per == 0) return cudaSuccess;
+  for (int b0 = 0; b0 < n; b0 += kMaxFillBufs) {
+    const int m = n - b0 < kMaxFillBufs ? n - b0 : kMaxFillBufs;
+    FillList L{};
+    for (int i = 0; i < m; i++) L.base[i] = bufs[b0 + i];
+    long long nb = (per + 255) / 256;
+    const long long cap = (148LL * 16 + m - 1) / m;   // ~16 CTAs per SM over all buffers
+    dim3 grid(unsigned(nb < cap ? nb : cap), unsigned(m));
+    if (es == 4) fill_xy_multi<float><<<grid, 256, 0, s>>>(L, g, px, py);
+    else fill_xy_multi<double><<<grid, 256, 0, s>>>(L, g, px, py);
   }
   return cudaGetLastError();
 }

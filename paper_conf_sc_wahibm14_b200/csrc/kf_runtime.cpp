@@ -309,11 +309,32 @@ static void run_fill(kf_exec* E, int buf, cudaStream_t s) {
     if (p.bc[a] == KF_BC_PERIODIC) CK(launch_fill(a, buf_ptr(E, buf), p.es, gm, s));
 }
 
+// Consecutive fills of a schedule in one launch (x and y together; z, if periodic, after them).
+static void run_fills(kf_exec* E, const std::vector<int>& bufs, cudaStream_t s) {
+  if (bufs.empty()) return;
+  const Program& p = E->prog->p;
+  Geom gm = geom(p);
+  if (getenv("KF_FILL_SINGLE")) {   // A/B switch: one launch per buffer and axis
+    for (int b : bufs) run_fill(E, b, s);
+    return;
+  }
+  std::vector<void*> ptr;
+  for (int b : bufs) ptr.push_back(buf_ptr(E, b));
+  CK(launch_fill_xy_multi(ptr.data(), int(ptr.size()), p.bc[0] == KF_BC_PERIODIC, p.bc[1] == KF_BC_PERIODIC, p.es, gm, s));
+  if (p.bc[2] == KF_BC_PERIODIC)
+    for (void* b : ptr) CK(launch_fill(2, b, p.es, gm, s));
+}
+
 static void run_step(kf_exec* E, int par, cudaStream_t s) {
+  std::vector<int> pend;
   for (const Op& op : E->sched[par]) {
     if (op.kind == 0) {
-      run_fill(E, op.buf, s);
-    } else if (E->profiling) {
+      pend.push_back(op.buf);
+      continue;
+    }
+    run_fills(E, pend, s);
+    pend.clear();
+    if (E->profiling) {
       cudaEvent_t a, b;
       if (E->evpool.size() >= 2) {
         a = E->evpool.back(); E->evpool.pop_back();
@@ -331,6 +352,7 @@ static void run_step(kf_exec* E, int par, cudaStream_t s) {
       launch_group(E, op.group, par, s);
     }
   }
+  run_fills(E, pend, s);
 }
 
 static void ensure_device(kf_exec* E) {
@@ -456,7 +478,7 @@ static void exec_run(kf_exec* E, void* const* arrays, void* scratch, uint64_t sc
     E->shell_init_scratch = scratch;
     E->shell_init_arrays = arr;
   }
-  for (int b : E->fill_all) run_fill(E, b, s);
+  run_fills(E, E->fill_all, s);
   int64_t reps = nsteps / E->period, rem = nsteps % E->period;
   if (E->use_graph && !E->profiling && reps > 0) {
     if (!E->gexec) {
@@ -643,12 +665,26 @@ kf_status kf_exec_get_info(const kf_exec* ex, kf_exec_info* out) {
     const Program& p = ex->prog->p;
     int naxes = 0;
     for (int a = 0; a < 3; a++) naxes += p.bc[a] == KF_BC_PERIODIC;
-    for (auto& sc : ex->sched)
+    // fill launches: one per run of consecutive fills (x and y batched, kMaxFillBufs buffers per
+    // launch) plus one per buffer for a periodic z axis; KF_FILL_SINGLE: one per buffer and axis
+    const bool single = getenv("KF_FILL_SINGLE") != nullptr;
+    const int nxy = (p.bc[0] == KF_BC_PERIODIC) + (p.bc[1] == KF_BC_PERIODIC);
+    for (auto& sc : ex->sched) {
+      int run = 0;
+      auto flush = [&]() {
+        if (run == 0) return;
+        fills += single ? run * naxes : (nxy ? (run + kMaxFillBufs - 1) / kMaxFillBufs : 0) +
+                                            (p.bc[2] == KF_BC_PERIODIC ? run : 0);
+        run = 0;
+      };
       for (auto& op : sc) {
-        if (op.kind == 0) fills += 1;
-        else launches += 1;
+        if (op.kind == 0) { run++; continue; }
+        flush();
+        launches += 1;
       }
-    r.fills_per_step = fills * naxes / ex->period;
+      flush();
+    }
+    r.fills_per_step = fills / ex->period;
     r.launches_per_step = launches / ex->period + r.fills_per_step;
     r.period = ex->period;
     r.compulsory_bytes_per_step = ex->step_bytes;
