@@ -347,6 +347,13 @@ kf_status kf_dist_create(kf_exec* const* parts, int32_t n_parts, int32_t px, int
  * if the plan needs none), each >= kf_exec_scratch_bytes.  Asynchronous on cuda_stream. */
 kf_status kf_dist_run(kf_dist* d, void* const* arrays, void* const* scratch, uint64_t scratch_bytes, int64_t nsteps,
                       const double* params, void* cuda_stream);
+/* Overlap of halo exchange with interior compute (default on): before a group that needs fresh
+ * ghosts, the exchanges run on an internal second stream (ordered after all work issued on
+ * cuda_stream) while the group's interior tiles -- those at least one ghost width inside the
+ * local domain in x and y, which read no ghost and write no exchanged strip -- run on
+ * cuda_stream; the other tiles are launched after the exchanges complete.  Results are
+ * identical either way; off = exchanges and whole-group launches in stream order. */
+kf_status kf_dist_set_overlap(kf_dist* d, int32_t on);
 void kf_dist_destroy(kf_dist* d);
 
 /* ------------------------------------------------------------------ utilities */

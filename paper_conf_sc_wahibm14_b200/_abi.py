@@ -150,6 +150,7 @@ SIGNATURES = {
     "kf_dist_create": (C.c_int, [C.POINTER(P), C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.c_int32,
                                  C.POINTER(C.c_uint8), C.POINTER(P)]),
     "kf_dist_run": (C.c_int, [P, C.POINTER(P), C.POINTER(P), C.c_uint64, C.c_int64, C.POINTER(C.c_double), P]),
+    "kf_dist_set_overlap": (C.c_int, [P, C.c_int32]),
     "kf_dist_destroy": (None, [P]),
     "kf_jit_check": (C.c_int, [P, I32P, C.POINTER(kf_target), C.c_int32, I32P, I32P, C.c_char_p, C.c_int64]),
 }

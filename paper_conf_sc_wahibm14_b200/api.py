@@ -325,6 +325,10 @@ class Dist:
             lib().kf_dist_destroy(h)
             self.h = None
 
+    def set_overlap(self, on: bool):
+        """Exchange / interior-compute overlap (kf_dist_set_overlap; default on)."""
+        check(lib().kf_dist_set_overlap(self.h, 1 if on else 0))
+
     def run(self, part_tensors, part_scratch, nsteps: int, params=None, stream=None):
         import torch
         stream = stream or torch.cuda.current_stream()

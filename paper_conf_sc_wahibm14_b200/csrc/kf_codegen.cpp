@@ -24,6 +24,27 @@
 
 namespace kf {
 
+// Tile rectangle [ix0, ix1) x [iy0, iy1) whose tiles lie at least the ghost width inside the
+// local domain on x and y (a11: they run while a halo exchange is in flight).
+Split split_units(const Program& p, const GroupLowering& L) {
+  Split s;
+  const int TX = L.tile[0], TY = L.tile[1];
+  const int NTX = int((p.n[0] + TX - 1) / TX), NTY = int((p.n[1] + TY - 1) / TY);
+  const int gx = p.ghost[0], gy = p.ghost[1];
+  s.ix0 = (gx + TX - 1) / TX;
+  s.iy0 = (gy + TY - 1) / TY;
+  s.ix1 = p.n[0] - gx - TX >= 0 ? int((p.n[0] - gx - TX) / TX) + 1 : 0;
+  s.iy1 = p.n[1] - gy - TY >= 0 ? int((p.n[1] - gy - TY) / TY) + 1 : 0;
+  s.ix1 = std::min(s.ix1, NTX);
+  s.iy1 = std::min(s.iy1, NTY);
+  s.ok = s.ix1 > s.ix0 && s.iy1 > s.iy0 && (s.ix1 - s.ix0) * (s.iy1 - s.iy0) < NTX * NTY;
+  const int TZ = L.tile[2] > 0 ? std::min<int>(L.tile[2], int(p.n[2])) : int(p.n[2]);
+  const int NTZ = int((p.n[2] + TZ - 1) / TZ);
+  s.interior_units = s.ok ? (s.ix1 - s.ix0) * (s.iy1 - s.iy0) * NTZ : 0;
+  s.boundary_units = s.ok ? NTX * NTY * NTZ - s.interior_units : 0;
+  return s;
+}
+
 static std::string lit(double v, int dtype) {
   char buf[64];
   if (dtype == KF_F32) {
@@ -117,6 +138,7 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
   o << "  real* out[" << std::max<size_t>(1, L.live_out.size()) << "];\n";
   o << "  const real* gsrc[" << std::max<size_t>(1, mid_rings.size()) << "];\n";
   o << "  double prm[" << std::max(1, p.n_params) << "];\n";
+  o << "  int mode, pad_;   // units: 0 all, 1 interior tiles only, 2 the others (kf_split_units)\n";
   o << "};\n";
   // register cap (__maxnreg__): at most what keeps the shared-memory-limited number of CTAs per SM
   // resident (minblocks 0; or minblocks CTAs) and never above the resource model's estimate R_est
@@ -137,7 +159,28 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
   o << "  unsigned char* sm = kf_smem_raw + ((128u - (kf_smem_u32(kf_smem_raw) & 127u)) & 127u);\n";
   o << "  u64* mbar = (u64*)(sm + " << L.mbar_off << ");\n";
   o << "  const int tid = threadIdx.x;\n";
-  o << "  int u = blockIdx.x;\n";
+  // interior / boundary unit split (a11 overlap): interior tiles lie >= the ghost width inside the
+  // local domain on x and y, so they neither read ghosts nor write the strips an exchange packs
+  {
+    const Split sp = split_units(p, L);
+    o << "  int u = blockIdx.x;\n";
+    if (sp.ok) {
+      const int IW = sp.ix1 - sp.ix0, IH = sp.iy1 - sp.iy0;
+      o << "  if (a.mode == 1) {\n"
+        << "    const int tz = u / " << IW * IH << ", r = u - tz * " << IW * IH << ";\n"
+        << "    u = (tz * NTY + " << sp.iy0 << " + r / " << IW << ") * NTX + " << sp.ix0 << " + r % " << IW << ";\n"
+        << "  } else if (a.mode == 2) {\n"
+        << "    const int nb = NTX * NTY - " << IW * IH << ", tz = u / nb;\n"
+        << "    int b = u - tz * nb, tx, ty;\n"
+        << "    if (b < " << sp.iy0 << " * NTX) { ty = b / NTX; tx = b % NTX; }\n"
+        << "    else if ((b -= " << sp.iy0 << " * NTX) < " << IH * (NTX - IW) << ") {\n"
+        << "      ty = " << sp.iy0 << " + b / " << NTX - IW << "; const int c = b % " << NTX - IW << "; tx = c < " << sp.ix0
+        << " ? c : c + " << IW << ";\n"
+        << "    } else { b -= " << IH * (NTX - IW) << "; ty = " << sp.iy1 << " + b / NTX; tx = b % NTX; }\n"
+        << "    u = (tz * NTY + ty) * NTX + tx;\n"
+        << "  }\n";
+    }
+  }
   o << "  const int x0 = (u % NTX) * TX; u /= NTX;\n";
   o << "  const int y0 = (u % NTY) * TY; u /= NTY;\n";
   o << "  const int z0 = u * TZ;\n";
@@ -546,6 +589,12 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
     }
     canvas_bounds = "  const bool cfxy = " + cxy + ";\n  const int cf0 = cfxy ? " + lo + " : 0, cf1 = cfxy ? " + hi + " : 0;\n";
   }
+  // rotated slot offsets are loop-carried uniform registers: with many ring slots they spill into
+  // vector registers (a 35-kernel group: 66 -> 88 registers), so large groups keep the counters
+  int rot_slots = 0;
+  for (const Ring& R : L.rings) rot_slots += R.slots > 1 ? R.slots : 0;
+  const bool rotate = rot_slots <= 32 && !getenv("KF_SLOT_COUNTERS");   // A/B switch: per-ring counters + kf_slot
+  if (getenv("KF_DEBUG")) fprintf(stderr, "codegen %s: %d rotated ring slots%s\n", cg.name.c_str(), rot_slots, rotate ? "" : " (counters)");
   auto emit_body = [&](int j) {
   o << "    if (tid == 0 && t + " << U << " * (NSTAGE - 1) < t1) issue(t + " << U << " * (NSTAGE - 1));\n";
   o << "    kf_mbar_wait(&mbar[((t - t0) / " << U << ") % NSTAGE], (((t - t0) / " << U << ") / NSTAGE) & 1);\n";
@@ -581,7 +630,9 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
     // unrolling: compile-time constants
     for (auto& [ring, om] : need) {
       const Ring& R = L.rings[ring];
-      if (j < 0)   // computed once per iteration (measured slightly faster than per-use macros)
+      if (j < 0 && rotate)   // slot offsets rotated at the end of every iteration
+        o << "    real* P" << ring << "_" << om << " = (real*)(sm + so" << ring << "_" << om << ");\n";
+      else if (j < 0)   // computed once per iteration (measured slightly faster than per-use macros)
         o << "    real* P" << ring << "_" << om << " = (real*)(sm + " << R.smem_off << " + kf_slot(cs" << ring << ", " << om
           << ", " << R.slots << ") * " << R.plane_bytes << ");\n";
       else
@@ -996,7 +1047,26 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
       for (auto& [key, src] : carry) o << "  real " << key_name("cq", key, "_r" + std::to_string(r)) << " = 0;\n";
   }
   o << canvas_bounds;
-  if (NU == 0) {
+  if (NU == 0 && rotate) {
+    // slot byte offsets of every ring, rotated by U slots per iteration: slot (c + om) mod n of a
+    // per-ring counter c costs ~5 uniform instructions per pointer and iteration (ncu: ~35 % of all
+    // instructions were uniform-datapath bookkeeping), a rotation one move per slot
+    for (size_t ri = 0; ri < L.rings.size(); ri++)
+      for (int sl = 0; sl < L.rings[ri].slots; sl++)
+        o << "  u32 so" << ri << "_" << sl << " = " << L.rings[ri].smem_off + sl * L.rings[ri].plane_bytes << "u;\n";
+    o << "  for (int t = t0; t < t1; t += " << U << ") {\n";
+    emit_body(-1);
+    for (size_t ri = 0; ri < L.rings.size(); ri++) {
+      const int n = L.rings[ri].slots;
+      if (n == 1 || U % n == 0) continue;
+      o << "    { const u32";
+      for (int sl = 0; sl < n; sl++) o << (sl ? ", " : " ") << "r" << sl << " = so" << ri << "_" << sl;
+      o << ";";
+      for (int sl = 0; sl < n; sl++) o << " so" << ri << "_" << sl << " = r" << (sl + U) % n << ";";
+      o << " }\n";
+    }
+    o << "  }\n";
+  } else if (NU == 0) {
     for (size_t ri = 0; ri < L.rings.size(); ri++) o << "  int cs" << ri << " = 0;\n";
     o << "  for (int t = t0; t < t1; t += " << U << ") {\n";
     emit_body(-1);

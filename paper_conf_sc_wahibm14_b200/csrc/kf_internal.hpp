@@ -115,6 +115,10 @@ struct Ring {
   int smem_off = 0;       // byte offset in dynamic SMEM
 };
 
+struct GroupLowering;
+// a11 overlap: the tile rectangle at least one ghost width inside the local domain (x, y)
+struct Split { bool ok = false; int ix0 = 0, ix1 = 0, iy0 = 0, iy1 = 0; int interior_units = 0, boundary_units = 0; };
+
 struct GroupLowering {
   std::vector<int> kernels;               // program order
   std::map<int, Ext> ext;                 // per kernel
@@ -185,6 +189,7 @@ struct Codegen {
   std::string name;
 };
 Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid);
+Split split_units(const Program& p, const GroupLowering& L);
 
 }  // namespace kf
 

@@ -151,6 +151,7 @@ struct GroupExec {
   CUmodule mod = nullptr;
   CUfunction fn = nullptr;
   int grid = 0, smem = 0, regs = -1, local = -1;
+  Split split;   // interior / boundary units (a11 overlap)
   uint64_t bytes = 0;
   std::vector<Ver> ins, outs, mids;
   size_t blob_size = 0;
@@ -243,7 +244,7 @@ static void build_blobs(kf_exec* E) {
     for (auto& g : E->G) {
       size_t ni = std::max<size_t>(1, g.ins.size()), no = std::max<size_t>(1, g.outs.size()),
              nm = std::max<size_t>(1, g.mids.size()), np = std::max(1, p.n_params);
-      size_t sz = 128 * ni + 8 * (no + nm + np);
+      size_t sz = 128 * ni + 8 * (no + nm + np) + 8;   // + int mode, pad (zero: every unit)
       sz = (sz + 63) / 64 * 64;
       g.blob_size = sz;
       std::vector<unsigned char> b(sz + 64, 0);
@@ -285,20 +286,32 @@ static void build_blobs(kf_exec* E) {
   E->blobs_valid = true;
 }
 
-static void launch_group(kf_exec* E, int gi, int par, cudaStream_t s) {
+// mode 0: every unit; 1: interior tiles only; 2: the other tiles (the group's Split)
+static void launch_group(kf_exec* E, int gi, int par, cudaStream_t s, int mode = 0) {
   GroupExec& g = E->G[gi];
   std::vector<unsigned char>& blob = E->blobs[par][gi];
   // The argument block is one __grid_constant__ struct; the driver copies it at launch.
   alignas(64) unsigned char tmp[32768];
   if (blob.size() > sizeof(tmp)) fail(KF_E_RESOURCE, "kernel argument block too large");
   std::memcpy(tmp, blob.data(), blob.size());
+  int grid = g.grid;
+  if (mode != 0) {
+    if (!g.split.ok) fail(KF_E_ARG, "group has no interior/boundary split");
+    grid = mode == 1 ? g.split.interior_units : g.split.boundary_units;
+    const size_t off = 128 * std::max<size_t>(1, g.ins.size()) +
+                       8 * (std::max<size_t>(1, g.outs.size()) + std::max<size_t>(1, g.mids.size()) +
+                            std::max(1, E->prog->p.n_params));
+    const int32_t m = mode;
+    std::memcpy(tmp + off, &m, 4);
+    if (grid == 0) return;
+  }
   void* params[] = {tmp};
   if (getenv("KF_DEBUG")) {
     fprintf(stderr, "launch %s grid=%d threads=%d smem=%d blob=%zu:", g.cg.name.c_str(), g.grid, g.L.threads, g.smem, blob.size());
     for (size_t i = 0; i < blob.size(); i += 8) fprintf(stderr, " %016llx", *(unsigned long long*)(tmp + i));
     fprintf(stderr, "\n");
   }
-  ckd(drv().launchKernel(g.fn, g.grid, 1, 1, g.L.threads, 1, 1, g.smem, (CUstream)s, params, nullptr),
+  ckd(drv().launchKernel(g.fn, grid, 1, 1, g.L.threads, 1, 1, g.smem, (CUstream)s, params, nullptr),
       ("cuLaunchKernel " + g.cg.name).c_str());
 }
 
@@ -566,6 +579,7 @@ kf_status kf_exec_create_ex(kf_program* prog, const int32_t* plan, const kf_targ
       g.L = std::move(Ls[gi]);
       g.cg = generate_group_kernel(p, g.L, gi);
       g.grid = int(units);
+      g.split = split_units(p, g.L);
       g.smem = g.L.smem;
       uint64_t rd, wr;
       g.bytes = group_bytes(p, E->plan.groups[gi], &rd, &wr);
@@ -860,6 +874,11 @@ struct kf_dist {
   void* comm = nullptr;
   void* stage = nullptr;         // NCCL staging (device): 4 strips of the largest face
   uint64_t stage_bytes = 0;
+  // overlap (a11): exchanges on a second stream while the group's interior tiles run
+  int overlap = 1;
+  cudaStream_t xs = nullptr;
+  cudaEvent_t ev_ready = nullptr, ev_done = nullptr;
+  int xs_device = -1;
 };
 
 namespace kf {
@@ -984,12 +1003,39 @@ static void dist_run(kf_dist* D, void* const* arrays, void* const* scratch, uint
   }
   kf_exec* E0 = D->parts[0];
   for (int b : E0->fill_all) dist_exchange(D, b, s);
+  if (D->overlap && !D->xs) {
+    CK(cudaGetDevice(&D->xs_device));
+    CK(cudaStreamCreateWithFlags(&D->xs, cudaStreamNonBlocking));
+    CK(cudaEventCreateWithFlags(&D->ev_ready, cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&D->ev_done, cudaEventDisableTiming));
+  }
+  std::vector<int> pend;   // exchanges due before the next group
   for (int64_t step = 0; step < nsteps; step++) {
     const int par = int(step % E0->period);
     for (const Op& op : E0->sched_full[par]) {
       if (op.kind == 0) {
-        dist_exchange(D, op.buf, s);
-      } else {
+        pend.push_back(op.buf);
+        continue;
+      }
+      // Overlap: the exchanges run on a second stream, ordered after everything
+      // issued so far, while the group's interior tiles -- at least one ghost width inside the
+      // local domain, so they read no ghost and write no strip an exchange packs -- run on the
+      // compute stream; the remaining tiles wait for the exchanges.
+      const bool split = D->overlap && !pend.empty() && E0->G[op.group].split.ok && !E0->profiling;
+      if (split) {
+        CK(cudaEventRecord(D->ev_ready, s));
+        CK(cudaStreamWaitEvent(D->xs, D->ev_ready, 0));
+        for (int b : pend) dist_exchange(D, b, D->xs);
+        CK(cudaEventRecord(D->ev_done, D->xs));
+        for (kf_exec* E : D->parts) launch_group(E, op.group, par, s, 1);
+        CK(cudaStreamWaitEvent(s, D->ev_done, 0));
+        for (kf_exec* E : D->parts) launch_group(E, op.group, par, s, 2);
+        pend.clear();
+        continue;
+      }
+      for (int b : pend) dist_exchange(D, b, s);
+      pend.clear();
+      {
         for (kf_exec* E : D->parts) {
           if (!E->profiling) {
             launch_group(E, op.group, par, s);
@@ -1012,6 +1058,7 @@ static void dist_run(kf_dist* D, void* const* arrays, void* const* scratch, uint
       }
     }
   }
+  for (int b : pend) dist_exchange(D, b, s);
   if (E0->period == 2 && (nsteps % 2) == 1)
     for (kf_exec* E : D->parts)
       for (int x = 0; x < p.na; x++)
@@ -1097,11 +1144,21 @@ kf_status kf_dist_run(kf_dist* d, void* const* arrays, void* const* scratch, uin
   });
 }
 
+kf_status kf_dist_set_overlap(kf_dist* d, int32_t on) {
+  KF_TRY({
+    if (!d) fail(KF_E_ARG, "null dist");
+    d->overlap = on ? 1 : 0;
+  });
+}
+
 void kf_dist_destroy(kf_dist* d) {
   if (!d) return;
   try {
     if (d->comm && nccl().commDestroy) nccl().commDestroy(d->comm);
     if (d->stage) cudaFree(d->stage);
+    if (d->xs) cudaStreamDestroy(d->xs);
+    if (d->ev_ready) cudaEventDestroy(d->ev_ready);
+    if (d->ev_done) cudaEventDestroy(d->ev_done);
   } catch (...) {
   }
   delete d;

@@ -90,13 +90,14 @@ def test_gloo_two_ranks_host_logic():
 
 
 # ----------------------------------------------------------------------------------- GPU
-def _run_loopback(desc, plan, inputs, nsteps, px, py, target=None):
+def _run_loopback(desc, plan, inputs, nsteps, px, py, target=None, overlap=True):
     import torch
     import paper_conf_sc_wahibm14_b200 as kf
     parts_np, local = kf.split_domain(desc, inputs, px, py)
     prog = kf.Program(local)
     execs = [kf.Exec(prog, plan, target) for _ in range(px * py)]
     dist = kf.Dist(execs, px, py)
+    dist.set_overlap(overlap)
     dev = [kf.device_arrays(prog, part) for part in parts_np]
     sb = execs[0].scratch_bytes()
     scr = [torch.empty(sb, dtype=torch.uint8, device="cuda") if sb else None for _ in execs]
@@ -139,3 +140,23 @@ def test_loopback_random_periodic_programs():
         for plan in (legal[0], legal[-1]):
             got = _run_loopback(desc, plan, inputs, 2, 2, 3, kf.Target(tile=(8, 4, 0)))
             assert compare(desc, got, ref) == [], (seed, plan)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("overlap", [True, False])
+def test_loopback_overlap_interior_boundary_split(overlap):
+    """Exchange / interior-compute overlap: local sub-domains large enough that every
+    group splits into interior tiles (launched while the exchanges run on the second stream) and
+    boundary tiles (after them); bit-exact with the oracle with and without the overlap."""
+    torch = pytest.importorskip("torch")
+    if not torch.cuda.is_available():
+        pytest.skip("needs a GPU")
+    import paper_conf_sc_wahibm14_b200 as kf
+    desc = P.weather(n=(128, 96, 10))
+    inputs = D.inputs_for(desc, 12)
+    ref = interp.run(desc, inputs, 3)
+    tgt = kf.Target(tile=(16, 8, 0))
+    plans = [P.weather_hand_plan(desc), kf.Program(desc).search(kf.SEARCH_HGGA, tgt, seed=1)[0]]
+    for plan in plans:
+        got = _run_loopback(desc, plan, inputs, 3, 2, 2, tgt, overlap=overlap)
+        assert compare(desc, got, ref) == [], (overlap, plan)
