@@ -264,7 +264,8 @@ def cpu_baseline(name: str, budget_s: float = 12.0):
 AUTOTUNE_CANDIDATES = [  # (tile, stages, zunroll, ringunroll, minblocks, canvas_ld)
     ((32, 8, 64), 2, 1, 0, 0, 1), ((32, 8, 64), 2, 1, 0, -1, 1), ((32, 8, 64), 2, 1, 0, -1, 0), ((32, 8, 64), 2, 1, 0, 0, 0),
     ((32, 8, 32), 2, 1, 0, -1, 1), ((32, 8, 32), 2, 1, 0, 0, 0), ((32, 8, 0), 2, 1, 0, -1, 1), ((64, 4, 64), 2, 1, 0, 0, 1),
-    ((16, 12, 64), 2, 1, 0, 0, 1), ((32, 8, 64), 3, 1, 0, -1, 1), ((32, 8, 64), 2, 1, 1, -1, 1), ((32, 8, 64), 2, 2, 0, 0, 1)]
+    ((16, 12, 64), 2, 1, 0, 0, 1), ((32, 8, 64), 3, 1, 0, -1, 1), ((32, 8, 64), 2, 1, 1, -1, 1), ((32, 8, 64), 2, 2, 0, 0, 1),
+    ((64, 8, 64), 2, 2, 0, 0, 1)]   # z-unroll 2 on 64x8: the fastest for the fp32 suite groups (tools/ab.py)
 
 
 def autotune(prog, plan, dev, base_kw, steps=4):

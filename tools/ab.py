@@ -19,10 +19,25 @@ HGGA = [0, 0, 0, 1, 1, 1, 1, 1, 1, 2, 2, 2, 2, 2, 2, 0, 2, 0, 0, 0, 0, 1, 1, 1, 
 def main():
     variants = json.loads(sys.argv[1])
     which = sys.argv[2] if len(sys.argv) > 2 else "hgga"
-    desc = P.weather(n=(512, 512, 128))
+    wl = sys.argv[3] if len(sys.argv) > 3 else "weather"
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    import bench
+    desc, gen, tkw, _ = bench.workload(wl)
     prog = kf.Program(desc)
-    plan = {"hgga": HGGA, "hand": P.weather_hand_plan(desc), "unfused": list(range(44))}.get(which) or json.loads(which)
-    dev = kf.device_arrays(prog, D.weather_inputs(desc, 3))
+    if which == "best":
+        plan = bench.choose_plan(prog, kf.Target(**tkw), "best")[0]
+    elif wl == "weather":
+        plan = {"hgga": HGGA, "hand": P.weather_hand_plan(desc), "unfused": list(range(44))}.get(which) or json.loads(which)
+    else:
+        plan = list(range(prog.nk)) if which == "unfused" else json.loads(which)
+    if gen is None:
+        L = prog.layout()
+        g = torch.Generator(device="cuda").manual_seed(3)
+        dt = torch.float64 if desc.dtype == 1 else torch.float32
+        dev = [torch.rand(L.elems, generator=g, device="cuda", dtype=dt) * 2 - 1 for _ in desc.arrays]
+    else:
+        dev = kf.device_arrays(prog, gen(desc, 3))
+    print(json.dumps({"workload": wl, "plan": plan}), flush=True)
     steps = 10
     for v in variants:
         saved = {}
