@@ -261,11 +261,13 @@ def cpu_baseline(name: str, budget_s: float = 12.0):
 
 
 # ---------------------------------------------------------------- GPU timing
-AUTOTUNE_CANDIDATES = [  # (tile, stages, zunroll, ringunroll, minblocks, canvas_ld)
+AUTOTUNE_CANDIDATES = [  # (tile, stages, zunroll, ringunroll, minblocks, canvas_ld[, pblock x])
     ((32, 8, 64), 2, 1, 0, 0, 1), ((32, 8, 64), 2, 1, 0, -1, 1), ((32, 8, 64), 2, 1, 0, -1, 0), ((32, 8, 64), 2, 1, 0, 0, 0),
     ((32, 8, 32), 2, 1, 0, -1, 1), ((32, 8, 32), 2, 1, 0, 0, 0), ((32, 8, 0), 2, 1, 0, -1, 1), ((64, 4, 64), 2, 1, 0, 0, 1),
     ((16, 12, 64), 2, 1, 0, 0, 1), ((32, 8, 64), 3, 1, 0, -1, 1), ((32, 8, 64), 2, 1, 1, -1, 1), ((32, 8, 64), 2, 2, 0, 0, 1),
-    ((64, 8, 64), 2, 2, 0, 0, 1)]   # z-unroll 2 on 64x8: the fastest for the fp32 suite groups (tools/ab.py)
+    ((64, 8, 64), 2, 2, 0, 0, 1),   # z-unroll 2 on 64x8: the fastest for the fp32 suite groups (tools/ab.py)
+    # canvas pairs (two x-adjacent points per thread, 16-byte vector shared loads/stores)
+    ((32, 8, 32), 2, 1, 0, -1, 1, 2), ((32, 8, 64), 2, 1, 0, -1, 0, 2), ((32, 8, 64), 2, 1, 0, 0, 1, 2)]
 
 
 def autotune(prog, plan, dev, base_kw, steps=4):
@@ -276,9 +278,11 @@ def autotune(prog, plan, dev, base_kw, steps=4):
     import paper_conf_sc_wahibm14_b200 as kf
     best = None
     tried = []
-    for tile, stages, zu, ru, mb, cl in AUTOTUNE_CANDIDATES:
+    for cand in AUTOTUNE_CANDIDATES:
+        tile, stages, zu, ru, mb, cl = cand[:6]
+        pb = cand[6] if len(cand) > 6 else 1
         kw = dict(base_kw)
-        kw.update(tile=tile, stages=stages, zunroll=zu, ringunroll=ru, minblocks=mb, canvas_ld=cl)
+        kw.update(tile=tile, stages=stages, zunroll=zu, ringunroll=ru, minblocks=mb, canvas_ld=cl, pblock=(pb, 1))
         tgt = kf.Target(**kw)
         try:
             ex = kf.Exec(prog, plan, tgt)
@@ -292,15 +296,15 @@ def autotune(prog, plan, dev, base_kw, steps=4):
         ex.run(dev, scr, steps)
         torch.cuda.synchronize()
         gms, _ = ex.group_times()
-        tried.append(((tile, stages, zu, ru, mb, cl), [g / steps for g in gms]))
+        tried.append((tuple(cand), [g / steps for g in gms]))
         if best is None:
             best = [(g / steps, kw) for g in gms]
         else:
             best = [min(b, (g / steps, kw), key=lambda v: v[0]) for b, g in zip(best, gms)]
         del ex, scr
     return ([kf.Target(**kw) for _, kw in best],
-            [(list(kw["tile"]), kw["stages"], kw["zunroll"], kw["ringunroll"], kw["minblocks"], kw["canvas_ld"])
-             for _, kw in best], tried)
+            [(list(kw["tile"]), kw["stages"], kw["zunroll"], kw["ringunroll"], kw["minblocks"], kw["canvas_ld"],
+              kw["pblock"][0]) for _, kw in best], tried)
 
 
 def max_over_ranks(x: float) -> float:
@@ -425,7 +429,8 @@ def run_kf(args):
         tuned = json.loads(args.tuned)
         gtargets = [kf.Target(**dict(tkw, tile=tuple(c[0]), stages=c[1], zunroll=c[2], ringunroll=c[3],
                                             minblocks=c[4] if len(c) > 4 else 0,
-                                            canvas_ld=c[5] if len(c) > 5 else 1))
+                                            canvas_ld=c[5] if len(c) > 5 else 1,
+                                            pblock=(c[6] if len(c) > 6 else 1, 1)))
                     for c in tuned]
     elif args.autotune:
         if rank == 0:
@@ -436,7 +441,8 @@ def run_kf(args):
             tuned = obj[0]
             gtargets = [kf.Target(**dict(tkw, tile=tuple(c[0]), stages=c[1], zunroll=c[2], ringunroll=c[3],
                                             minblocks=c[4] if len(c) > 4 else 0,
-                                            canvas_ld=c[5] if len(c) > 5 else 1))
+                                            canvas_ld=c[5] if len(c) > 5 else 1,
+                                            pblock=(c[6] if len(c) > 6 else 1, 1)))
                         for c in tuned]
     rn = Runner(prog, plan, target, gtargets, new_dist_info())
     jit_s = time.time() - t0
@@ -610,7 +616,7 @@ def main():
     ap.add_argument("--autotune", type=int, default=1, help="per-group launch configuration by measurement (1/0)")
     ap.add_argument("--tuned", default=None, help="JSON per-group configs [[tile,stages,zunroll,ringunroll(,minblocks)],...] "
                                                   "(skips autotune; as printed in config.per_group_launch_config: "
-                                                  "[tile, stages, zunroll, ringunroll, minblocks, canvas_ld])")
+                                                  "[tile, stages, zunroll, ringunroll, minblocks, canvas_ld, pblock_x])")
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "kf":
         args.warmup = 3

@@ -56,6 +56,16 @@ CanvasPlan plan_canvas(const Program& p, const GroupLowering& L) {
   // one canvas point per thread only: with several rounds the forwarded values of all rounds stay
   // live together (register pressure), and the per-kernel fast path is used instead
   c.ok = !alive.empty() && L.pblock[0] == 1 && L.pblock[1] == 1 && c.rounds == 1 && !getenv("KF_NO_CANVAS");
+  // pair mode: pairs aligned to even tile-relative x (TX and NX even), so a pair never straddles
+  // the tile or domain edge; one pair per thread
+  if (!alive.empty() && L.pblock[0] == 2 && L.pblock[1] == 1 && U == 1 && TX % 2 == 0 && p.n[0] % 2 == 0 &&
+      !L.ghost_write && !getenv("KF_NO_CANVAS")) {
+    c.lop = (c.clo[0] + 1) / 2;
+    c.hip = (c.chi[0] + 1) / 2;
+    c.cwp = TX / 2 + c.lop + c.hip;
+    c.rounds = (c.cwp * c.ch + L.threads - 1) / L.threads;
+    c.pair = c.ok = c.rounds == 1;
+  }
   // versions whose every in-group read is forwarded need no shared-memory copy in fast iterations
   for (int k : alive)
     for (auto& [x, offs] : p.kernels[k].reads) {

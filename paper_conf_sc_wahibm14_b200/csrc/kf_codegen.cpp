@@ -127,6 +127,7 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
   for (int k : L.kernels) o << " " << p.kernels[k].name;
   o << "\n" << kPrelude;
   o << "typedef " << real << " real;\n";
+  o << "typedef " << (p.dtype == KF_F32 ? "float2" : "double2") << " real2;\n";
   o << "#define NX " << NX << "\n#define NY " << NY << "\n#define NZ " << NZ << "\n";
   o << "#define GX " << p.ghost[0] << "\n#define GY " << p.ghost[1] << "\n#define GZ " << p.ghost[2] << "\n";
   o << "#define PITCH " << lay.pitch << "ll\n#define PLANE " << lay.plane << "ll\n#define XOFF " << lay.xoff << "\n";
@@ -206,7 +207,34 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
   const bool canvas_mode = cv.ok;
   std::set<int> canvas_pitches;
   for (auto& r : L.rings) canvas_pitches.insert(r.px);
-  if (canvas_mode)
+  const bool pair_mode = canvas_mode && cv.pair;
+  const int PSH = 2 * cv.lop - clo[0];   // pair mode: canvas x of the thread's first point = 2 * pair column - PSH
+  if (pair_mode) {
+    // pair mode: row-aligned threads over the tile's TX/2 pair columns, then the halo pair columns
+    // (column-major); cx = canvas x of the first point (even tile-relative x: pairs are 16-byte
+    // aligned in every ring row and in HBM)
+    const int TXp = TX / 2, LP = cv.lop, CWp = cv.cwp;
+    o << "  int cxp_r0, cy_r0;\n";
+    o << "  if (tid < " << TXp * CH << ") { cy_r0 = tid / " << TXp << "; cxp_r0 = " << LP << " + tid - cy_r0 * " << TXp << "; }\n";
+    o << "  else { const int s = tid - " << TXp * CH << ", c = s / " << CH << "; cy_r0 = s - c * " << CH << "; cxp_r0 = c < " << LP
+      << " ? c : c + " << TXp << "; }\n";
+    o << "  const bool ca_r0 = tid < " << CWp * CH << ";\n";
+    o << "  if (!ca_r0) { cxp_r0 = " << LP << "; cy_r0 = 0; }   // in bounds for unpredicated loads\n";
+    o << "  const int cx_r0 = 2 * cxp_r0 - " << PSH << ";\n";
+    for (int pch : canvas_pitches) o << "  const int cb" << pch << "_r0 = cy_r0 * " << pch << " + cx_r0;\n";
+    o << "  const int cgx_r0 = x0 + cx_r0 - " << clo[0] << ", cgy_r0 = y0 + cy_r0 - " << clo[1] << ";\n";
+    o << "  const bool cT_r0 = ca_r0 && cx_r0 >= " << clo[0] << " && cx_r0 < " << clo[0] + TX << " && cy_r0 >= " << clo[1]
+      << " && cy_r0 < " << clo[1] + TY << " && cgx_r0 < NX && cgy_r0 < NY;\n";
+    for (int k : alive) {
+      const Ext& e = L.ext.at(k);
+      const int ox = clo[0] - e.elo[0], oy = clo[1] - e.elo[1];
+      const int WX = TX + e.elo[0] + e.ehi[0], WY = TY + e.elo[1] + e.ehi[1];
+      for (int j = 0; j < 2; j++)
+        o << "  const bool ce" << k << "_" << j << " = ca_r0 && cx_r0 + " << j << " >= " << ox << " && cx_r0 + " << j << " < "
+          << ox + WX << " && cy_r0 >= " << oy << " && cy_r0 < " << oy + WY << ";\n";
+    }
+  }
+  if (canvas_mode && !pair_mode)
     for (int r = 0; r < CROUNDS; r++) {
       const std::string rs = "_r" + std::to_string(r);
       o << "  const int ci" << rs << " = tid + " << r * NT << ";\n";
@@ -382,7 +410,7 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
   // slow iteration they are reloaded.  carry[key] = source: a load key or a forwarded value.
   struct Src { bool is_load; Key key; int x, v, uu; };
   std::map<Key, Src> carry;
-  if (canvas_mode && getenv("KF_CQ")) {   // off by default: the carried registers cost occupancy (measured slower)
+  if (canvas_mode && !pair_mode && getenv("KF_CQ")) {   // off by default: the carried registers cost occupancy (measured slower)
     // widen the load predicate of (ring, po + U, off) to cover (ring, po, off): both lie in the
     // ring's box at every plane, and the wider load then feeds the next iteration's narrower read
     for (auto& [key, rc] : krect) {
@@ -564,6 +592,155 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
       }
     }
     if (!carry.empty()) o << "      cqv = true;\n";
+  };
+  // Pair mode (cv.pair): the same phases, forwarding and load CSE as emit_canvas, for two
+  // x-adjacent points per thread.  A shared value is loaded as part of the 16-byte-aligned pair
+  // (2 elements) containing it, one vector load per distinct (ring, plane, pair offset) in a phase:
+  // a 4th-order x stencil on a point pair needs 3 vector loads instead of 8 scalar ones.  Ring and
+  // live-out stores are vector stores where the pair is aligned.  U = 1, no z-queue carries.
+  auto mod2 = [](int v) { return ((v % 2) + 2) % 2; };
+  auto emit_canvas_pairs = [&]() {
+    const int CWp = cv.cwp;
+    using PK = std::tuple<int, int, int>;   // ring, plane offset, element offset of the aligned pair
+    std::map<std::tuple<int, int, int>, std::string> fwd;   // (x, v, point) -> value
+    auto pk_of = [&](int k, int x, const Off& d, int j, int* comp) {
+      const Key key = load_key(k, x, d, 0);
+      const int e = key.off + j;
+      *comp = mod2(PSH + e);   // parity of the absolute element index (row pitches are even)
+      return PK{key.ring, key.po, e - *comp};
+    };
+    for (size_t ph = 0; ph < cph.size(); ph++) {
+      if (ph > 0) o << "      __syncthreads();\n";
+      // lanes (first point's canvas x, row) needing each pair load in this phase
+      std::map<PK, Rect> prect;
+      for (int k : cph[ph])
+        for (auto& [x, offs] : p.kernels[k].reads)
+          for (auto& d : offs)
+            for (int j = 0; j < 2; j++) {
+              int pr, u2, comp;
+              if (fwd_src(k, x, d, 0, &pr, &u2)) continue;
+              const Rect rc = krect.at(load_key(k, x, d, 0));
+              const PK pk = pk_of(k, x, d, j, &comp);
+              const Rect rj{rc[0] - j, rc[1] - j, rc[2], rc[3]};
+              auto it = prect.find(pk);
+              if (it == prect.end()) prect[pk] = rj;
+              else {
+                auto& a = it->second;
+                a = {std::min(a[0], rj[0]), std::max(a[1], rj[1]), std::min(a[2], rj[2]), std::max(a[3], rj[3])};
+              }
+            }
+      std::map<PK, std::string> ldname;
+      std::vector<std::tuple<int, std::vector<std::string>, std::vector<std::string>>> done;   // (k, vals pt0, vals pt1)
+      for (int k : cph[ph]) {
+        const Kernel& K = p.kernels[k];
+        o << "      // kernel " << k << " " << K.name << " (canvas pairs)\n";
+        std::vector<std::string> vals[2];
+        for (int j = 0; j < 2; j++)
+          for (size_t si = 0; si < K.stmts.size(); si++) {
+            std::vector<std::string> st;
+            int tmp = 0;
+            for (const Insn& in : K.stmts[si].rpn) {
+              std::string t = "c" + std::to_string(k) + "s" + std::to_string(si) + "_" + std::to_string(tmp++) + "_p" + std::to_string(j);
+              std::string f;
+              switch (in.op) {
+                case KF_OP_CONST: f = lit(in.imm, p.dtype); break;
+                case KF_OP_PARAM: f = "(real)a.prm[" + std::to_string(in.arg) + "]"; break;
+                case KF_OP_LOAD: {
+                  int pr, u2, comp;
+                  if (fwd_src(k, in.arg, in.d, 0, &pr, &u2)) {
+                    f = fwd.at(std::make_tuple(in.arg, p.vr(k, in.arg), j));
+                    break;
+                  }
+                  const PK pk = pk_of(k, in.arg, in.d, j, &comp);
+                  auto it = ldname.find(pk);
+                  if (it == ldname.end()) {
+                    const auto& [ring, po, rel] = pk;
+                    const Ring& RR = L.rings[ring];
+                    const Rect& rc = prect.at(pk);
+                    const std::string nm = "pl" + std::to_string(ring) + "_" + (po < 0 ? "m" + std::to_string(-po) : std::to_string(po)) +
+                                           "_" + (rel < 0 ? "m" + std::to_string(-rel) : std::to_string(rel)) + "_h" + std::to_string(ph);
+                    const std::string acc = "*(const real2*)&P" + std::to_string(ring) + "_" + std::to_string(slot(ring, po)) + "[cb" +
+                                            std::to_string(RR.px) + "_r0 + " + std::to_string(rel) + "]";
+                    // every address the load can form (all pair columns, rows, ring slots) in the rings' SMEM?
+                    const long long cxmin = -PSH, cxmax = 2LL * (CWp - 1) - PSH;
+                    const long long amin = RR.smem_off + (cxmin + rel) * p.es;
+                    const long long amax = RR.smem_off + (long long)(RR.slots - 1) * RR.plane_bytes +
+                                           ((long long)(CH - 1) * RR.px + cxmax + rel + 2) * p.es;
+                    if (L.canvas_ld && amin >= 0 && amax <= L.mbar_off)
+                      o << "      const real2 " << nm << " = " << acc << ";\n";
+                    else
+                      o << "      const real2 " << nm << " = (ca_r0 && cx_r0 >= " << rc[0] << " && cx_r0 < " << rc[1] << " && cy_r0 >= " << rc[2]
+                        << " && cy_r0 < " << rc[3] << ") ? " << acc << " : real2{(real)0, (real)0};\n";
+                    it = ldname.emplace(pk, nm).first;
+                  }
+                  f = it->second + (comp ? ".y" : ".x");
+                  break;
+                }
+                case KF_OP_NEG: case KF_OP_ABS: case KF_OP_SQRT: {
+                  std::string a1 = st.back(); st.pop_back();
+                  f = in.op == KF_OP_NEG ? "-" + a1
+                    : in.op == KF_OP_ABS ? (p.dtype == KF_F32 ? "fabsf(" : "fabs(") + a1 + ")"
+                                         : (p.dtype == KF_F32 ? "sqrtf(" : "sqrt(") + a1 + ")";
+                  break;
+                }
+                default: {
+                  std::string b = st.back(); st.pop_back();
+                  std::string a1 = st.back(); st.pop_back();
+                  switch (in.op) {
+                    case KF_OP_ADD: f = a1 + " + " + b; break;
+                    case KF_OP_SUB: f = a1 + " - " + b; break;
+                    case KF_OP_MUL: f = a1 + " * " + b; break;
+                    case KF_OP_DIV: f = a1 + " / " + b; break;
+                    case KF_OP_MIN: f = "(" + b + " < " + a1 + ") ? " + b + " : " + a1; break;
+                    case KF_OP_MAX: f = "(" + a1 + " < " + b + ") ? " + b + " : " + a1; break;
+                  }
+                }
+              }
+              o << "      const real " << t << " = " << f << ";\n";
+              st.push_back(t);
+            }
+            vals[j].push_back(st.back());
+          }
+        for (int j = 0; j < 2; j++)
+          for (size_t si = 0; si < K.stmts.size(); si++)
+            fwd[std::make_tuple(K.stmts[si].out, p.vw(k, K.stmts[si].out), j)] = vals[j][si];
+        done.emplace_back(k, vals[0], vals[1]);
+      }
+      // stores of the phase (after all its loads)
+      for (auto& [k, v0, v1] : done) {
+        const Kernel& K = p.kernels[k];
+        const Ext& e = L.ext.at(k);
+        const int ox = clo[0] - e.elo[0], oy = clo[1] - e.elo[1];
+        const std::string c0 = "ce" + std::to_string(k) + "_0", c1 = "ce" + std::to_string(k) + "_1";
+        bool any_out = false;
+        for (size_t si = 0; si < K.stmts.size(); si++) {
+          const Ver v{K.stmts[si].out, p.vw(k, K.stmts[si].out)};
+          const int ring = L.ring_of(v);
+          if (ring >= 0 && need_sts.count(v)) {
+            const Ring& R = L.rings[ring];
+            const std::string base = "P" + std::to_string(ring) + "_" + std::to_string(slot(ring, -L.delay.at(k))) + "[cb" +
+                                     std::to_string(R.px) + "_r0 - " + std::to_string(oy * R.px + ox);
+            if (mod2(PSH + ox) == 0)   // the pair is aligned in this ring
+              o << "      if (" << c0 << " && " << c1 << ") *(real2*)&" << base << "] = real2{" << v0[si] << ", " << v1[si]
+                << "};\n      else { if (" << c0 << ") " << base << "] = " << v0[si] << "; if (" << c1 << ") " << base
+                << " + 1] = " << v1[si] << "; }\n";
+            else
+              o << "      if (" << c0 << ") " << base << "] = " << v0[si] << ";\n      if (" << c1 << ") " << base << " + 1] = " << v1[si]
+                << ";\n";
+          }
+          if (out_index(v) >= 0) any_out = true;
+        }
+        if (!any_out) continue;
+        const std::string pz = "(t - " + std::to_string(L.delay.at(k)) + ")";
+        o << "      if (cT_r0 && " << pz << " >= z0 && " << pz << " < z1) {\n";
+        o << "        const long long gi = (long long)" << pz << " * PLANE + (long long)cgy_r0 * PITCH + cgx_r0;\n";
+        for (size_t si = 0; si < K.stmts.size(); si++) {
+          const int oi = out_index(Ver{K.stmts[si].out, p.vw(k, K.stmts[si].out)});
+          if (oi >= 0) o << "        *(real2*)&a.out[" << oi << "][gi] = real2{" << v0[si] << ", " << v1[si] << "};\n";
+        }
+        o << "      }\n";
+      }
+    }
   };
   auto qname = [](int k, const std::string& ps, int ring, int dz) {
     return "q" + std::to_string(k) + ps + "_" + std::to_string(ring) + "_" + (dz < 0 ? "m" + std::to_string(-dz) : std::to_string(dz));
@@ -996,7 +1173,8 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
     }
     if (!getenv("KF_CANVAS_COND")) c = "t >= cf0 && t < cf1";   // A/B switch: the per-kernel conjunction
     o << "    if (" << c << ") {   // ---- fast iteration on the canvas\n";
-    emit_canvas();
+    if (pair_mode) emit_canvas_pairs();
+    else emit_canvas();
     o << "    } else {\n";
     if (!carry.empty()) o << "    cqv = false;\n";
   }

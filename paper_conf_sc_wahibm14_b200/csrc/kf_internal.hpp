@@ -177,6 +177,10 @@ struct CanvasPlan {
   std::vector<std::vector<int>> phases;   // kernels between barriers
   std::map<CanvasKey, Rect> krect; // shared loads and the rect of lanes that issue them
   double lds_bytes = 0, sts_bytes = 0, tma_bytes = 0;   // per fast iteration per U planes
+  // pair mode (pblock 2x1, U = 1): a thread owns two x-adjacent canvas points whose pair starts on
+  // an even (16-byte for fp64) element; shared loads/stores and live-out stores are 2-wide vectors
+  bool pair = false;
+  int lop = 0, hip = 0, cwp = 0;   // pair columns left of / right of the tile, per canvas row
 };
 bool canvas_forward(const Program& p, const GroupLowering& L, int k, int x, const Off& d, int uu, int* prod, int* up);
 CanvasKey canvas_key(const Program& p, const GroupLowering& L, const CanvasPlan& c, int k, int x, const Off& d, int uu);

@@ -224,9 +224,33 @@ def test_canvas_paths_random_programs(seed, monkeypatch):
         monkeypatch.setenv("KF_CQ", "1")
     tile = [(16, 8, 0), (8, 8, 7), (32, 4, 0), (16, 4, 9)][seed % 4]
     for plan in pick:
-        for skew, mb, zu, cl in ((0, 0, 1, 1), (0, 0, 1, 0), (1, -1, 1, 1), (seed % 2, 0, 2, seed % 2)):
-            got, _ = run_kf(desc, plan, inputs, nsteps, kf.Target(tile=tile, skew=skew, minblocks=mb, zunroll=zu, canvas_ld=cl))
-            assert compare(desc, got, ref) == [], (plan, tile, skew, mb, zu, cl)
+        for skew, mb, zu, cl, pb in ((0, 0, 1, 1, 1), (0, 0, 1, 0, 1), (1, -1, 1, 1, 1), (seed % 2, 0, 2, seed % 2, 1),
+                                     (0, 0, 1, 1, 2), (0, -1, 1, 0, 2)):
+            t = kf.Target(tile=tile, skew=skew, minblocks=mb, zunroll=zu, canvas_ld=cl, pblock=(pb, 1))
+            got, _ = run_kf(desc, plan, inputs, nsteps, t)
+            assert compare(desc, got, ref) == [], (plan, tile, skew, mb, zu, cl, pb)
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_canvas_pairs_random_programs(seed):
+    """Pair mode of the canvas (pblock 2x1: two x-adjacent points per thread, 16-byte vector shared
+    loads/stores and live-out stores) on random programs with even nx, every boundary condition mix,
+    both dtypes, predicated and unpredicated loads."""
+    rng = np.random.default_rng(5000 + seed)
+    bc = tuple(int(x) for x in rng.integers(0, 2, size=3))
+    flags = [0, PROG_RELAX_EXPANDABLE, PROG_RELAX_ALL][seed % 3]
+    dtype = DT_F64 if seed % 2 else DT_F32
+    n = (2 * int(rng.integers(8, 20)), int(rng.integers(10, 30)), int(rng.integers(6, 14)))
+    desc = P.random_program(6000 + seed, nk=6, na=4, n=n, dtype=dtype, bc=bc, flags=flags, max_r=1 + seed % 2)
+    inputs = D.uniform(desc, seed)
+    ref = interp.run(desc, inputs, 2)
+    legal = En.legal_plans(desc)
+    pick = sorted(legal, key=lambda p: len(set(p)))[:3]
+    tile = [(16, 8, 0), (8, 8, 5), (32, 4, 0)][seed % 3]
+    for plan in pick:
+        for cl in (0, 1):
+            got, _ = run_kf(desc, plan, inputs, 2, kf.Target(tile=tile, pblock=(2, 1), canvas_ld=cl))
+            assert compare(desc, got, ref) == [], (plan, tile, cl)
 
 
 @pytest.mark.parametrize("cq", [0, 1])
@@ -241,7 +265,8 @@ def test_canvas_weather_knobs(cq, monkeypatch):
     tgt = kf.Target(tile=(32, 8, 0))
     plans = [prog.search(kf.SEARCH_HGGA, tgt, seed=s)[0] for s in (1, 2)]
     for plan in plans:
-        for kw in (dict(), dict(canvas_ld=0), dict(skew=1), dict(minblocks=-1, ringunroll=1), dict(tile=(32, 8, 5))):
+        for kw in (dict(), dict(canvas_ld=0), dict(pblock=(2, 1)), dict(pblock=(2, 1), canvas_ld=0), dict(skew=1),
+                   dict(minblocks=-1, ringunroll=1), dict(tile=(32, 8, 5))):
             t = kf.Target(**dict(dict(tile=(32, 8, 0)), **kw))
             if kw and prog.validate(plan, t)[0] != 0:   # e.g. V7: skew / ring unrolling need more SMEM
                 continue
