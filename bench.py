@@ -424,7 +424,7 @@ def run_kf(args):
             obj = [(plan, plan_kind, candidates)]
             torch.distributed.broadcast_object_list(obj, 0)
             plan, plan_kind, candidates = obj[0]
-    tuned, gtargets = None, None
+    tuned, gtargets, tried = None, None, None
     if args.tuned:   # fixed per-group configs (e.g. for an ncu run of exactly the timed configuration)
         tuned = json.loads(args.tuned)
         gtargets = [kf.Target(**dict(tkw, tile=tuple(c[0]), stages=c[1], zunroll=c[2], ringunroll=c[3],
@@ -434,7 +434,7 @@ def run_kf(args):
                     for c in tuned]
     elif args.autotune:
         if rank == 0:
-            gtargets, tuned, _ = autotune(prog, plan, dev, tkw)
+            gtargets, tuned, tried = autotune(prog, plan, dev, tkw)
         if world > 1:
             obj = [tuned]
             torch.distributed.broadcast_object_list(obj, 0)
@@ -529,7 +529,9 @@ def run_kf(args):
                                    f"exchange, weak (512x512x128 per GPU)") if world > 1 else "1 GPU",
                    "graph": world == 1, "jit_s": round(jit_s, 2),
                    "per_group_launch_config": tuned if tuned else "uniform",
-                   "plan_candidates": candidates},
+                   "plan_candidates": candidates,
+                   "autotune_tried": [{"config": list(c), "group_ms": [round(x, 4) for x in g]} for c, g in tried]
+                   if tried else None},
         "hbm_gbs_compulsory": achieved_step,
         "frac_of_measured_copy": achieved_step / hbm_peak,
         "frac_of_nominal_8TBs": achieved_step / 8000.0,

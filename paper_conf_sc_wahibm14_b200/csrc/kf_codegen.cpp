@@ -599,16 +599,99 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
   // a 4th-order x stencil on a point pair needs 3 vector loads instead of 8 scalar ones.  Ring and
   // live-out stores are vector stores where the pair is aligned.  U = 1, no z-queue carries.
   auto mod2 = [](int v) { return ((v % 2) + 2) % 2; };
+  using PK = std::tuple<int, int, int>;   // ring, plane offset, element offset of the aligned pair
+  auto pk_of = [&](int k, int x, const Off& d, int j, int* comp) {
+    const Key key = load_key(k, x, d, 0);
+    const int e = key.off + j;
+    *comp = mod2(PSH + e);   // parity of the absolute element index (row pitches are even)
+    return PK{key.ring, key.po, e - *comp};
+  };
+  // lanes (first point's canvas x, row) needing each pair load over the whole fast iteration, and
+  // whether the load can be issued unpredicated (every address it can form lies in the rings)
+  std::map<PK, Rect> pall;
+  auto pair_nopred = [&](const PK& pk) {
+    const auto& [ring, po, rel] = pk;
+    const Ring& RR = L.rings[ring];
+    const long long cxmin = -PSH, cxmax = 2LL * (cv.cwp - 1) - PSH;
+    const long long amin = RR.smem_off + (cxmin + rel) * p.es;
+    const long long amax = RR.smem_off + (long long)(RR.slots - 1) * RR.plane_bytes +
+                           ((long long)(CH - 1) * RR.px + cxmax + rel + 2) * p.es;
+    return L.canvas_ld && amin >= 0 && amax <= L.mbar_off;
+  };
+  // z register queues of the pair canvas: a pair value (ring, po, rel) read at iteration t is the
+  // value (ring, po + 1, rel) had at iteration t - 1 -- loaded then by the same thread, or computed
+  // then by it (its own forwarded result one plane earlier).  Such values are carried in registers
+  // across fast iterations instead of re-read from shared memory (fp64: centre-column z stencils
+  // and the z-flux read at dz = -1); after a slow iteration they are reloaded once.
+  struct PSrc { bool is_load; PK src; int x, v; };
+  std::map<PK, PSrc> pcarry;
+  if (pair_mode) {
+    for (int k : alive)
+      for (auto& [x, offs] : p.kernels[k].reads)
+        for (auto& d : offs)
+          for (int j = 0; j < 2; j++) {
+            int pr, u2, comp;
+            if (fwd_src(k, x, d, 0, &pr, &u2)) continue;
+            const Rect rc = krect.at(load_key(k, x, d, 0));
+            const PK pk = pk_of(k, x, d, j, &comp);
+            const Rect rj{rc[0] - j, rc[1] - j, rc[2], rc[3]};
+            auto it = pall.find(pk);
+            if (it == pall.end()) pall[pk] = rj;
+            else {
+              auto& a = it->second;
+              a = {std::min(a[0], rj[0]), std::max(a[1], rj[1]), std::min(a[2], rj[2]), std::max(a[3], rj[3])};
+            }
+          }
+    if (!getenv("KF_PAIR_NO_CQ"))   // A/B switch
+      for (auto& [pk, rc] : pall) {
+        const auto& [ring, po, rel] = pk;
+        const PK nx{ring, po + 1, rel};
+        auto it = pall.find(nx);
+        if (it != pall.end()) {
+          const Rect& a = it->second;
+          const bool covers = pair_nopred(nx) || (a[0] <= rc[0] && a[1] >= rc[1] && a[2] <= rc[2] && a[3] >= rc[3]);
+          if (covers) pcarry[pk] = PSrc{true, nx, 0, 0};
+          continue;
+        }
+        // the thread's own result one plane earlier: an in-group ring, the pair of the thread's own
+        // points (element offset of the canvas point, aligned), computed at plane t + po + 1
+        const Ring& R = L.rings[ring];
+        if (R.live_in) continue;
+        const int off0 = (R.blo[1] - clo[1]) * R.px + (R.ax_lo - clo[0]);
+        const int pk_ = R.producer;
+        if (mod2(PSH + off0) != 0 || rel != off0 || po + 1 != -L.delay.at(pk_)) continue;
+        const Rect rp = canvas_rect(L, cv, pk_);   // the producer's region (first point's x, both points inside)
+        if (rp[0] <= rc[0] && rp[1] - 1 >= rc[1] && rp[2] <= rc[2] && rp[3] >= rc[3])
+          pcarry[pk] = PSrc{false, nx, R.ver.x, R.ver.v};
+      }
+  }
+  auto pq_name = [&](const PK& pk) {
+    const auto& [ring, po, rel] = pk;
+    return "pq" + std::to_string(ring) + "_" + (po < 0 ? "m" + std::to_string(-po) : std::to_string(po)) + "_" +
+           (rel < 0 ? "m" + std::to_string(-rel) : std::to_string(rel));
+  };
+  auto pair_acc = [&](const PK& pk) {
+    const auto& [ring, po, rel] = pk;
+    return "*(const real2*)&P" + std::to_string(ring) + "_" + std::to_string(slot(ring, po)) + "[cb" +
+           std::to_string(L.rings[ring].px) + "_r0 + " + std::to_string(rel) + "]";
+  };
+  auto pair_pred = [&](const Rect& rc) {
+    return "ca_r0 && cx_r0 >= " + std::to_string(rc[0]) + " && cx_r0 < " + std::to_string(rc[1]) + " && cy_r0 >= " +
+           std::to_string(rc[2]) + " && cy_r0 < " + std::to_string(rc[3]);
+  };
   auto emit_canvas_pairs = [&]() {
-    const int CWp = cv.cwp;
-    using PK = std::tuple<int, int, int>;   // ring, plane offset, element offset of the aligned pair
     std::map<std::tuple<int, int, int>, std::string> fwd;   // (x, v, point) -> value
-    auto pk_of = [&](int k, int x, const Off& d, int j, int* comp) {
-      const Key key = load_key(k, x, d, 0);
-      const int e = key.off + j;
-      *comp = mod2(PSH + e);   // parity of the absolute element index (row pitches are even)
-      return PK{key.ring, key.po, e - *comp};
-    };
+    std::map<PK, std::string> ldfirst_p;                     // first load of each pair key this iteration
+    // carried pair values: loaded once after a slow iteration
+    if (!pcarry.empty()) {
+      o << "      if (!pqv) {\n";
+      for (auto& [pk, src] : pcarry) {
+        const Rect& rc = pall.at(pk);
+        if (pair_nopred(pk)) o << "        " << pq_name(pk) << " = " << pair_acc(pk) << ";\n";
+        else o << "        " << pq_name(pk) << " = (" << pair_pred(rc) << ") ? " << pair_acc(pk) << " : real2{(real)0, (real)0};\n";
+      }
+      o << "      }\n";
+    }
     for (size_t ph = 0; ph < cph.size(); ph++) {
       if (ph > 0) o << "      __syncthreads();\n";
       // lanes (first point's canvas x, row) needing each pair load in this phase
@@ -652,26 +735,22 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
                     break;
                   }
                   const PK pk = pk_of(k, in.arg, in.d, j, &comp);
+                  if (pcarry.count(pk)) {
+                    f = pq_name(pk) + (comp ? ".y" : ".x");
+                    break;
+                  }
                   auto it = ldname.find(pk);
                   if (it == ldname.end()) {
                     const auto& [ring, po, rel] = pk;
-                    const Ring& RR = L.rings[ring];
                     const Rect& rc = prect.at(pk);
                     const std::string nm = "pl" + std::to_string(ring) + "_" + (po < 0 ? "m" + std::to_string(-po) : std::to_string(po)) +
                                            "_" + (rel < 0 ? "m" + std::to_string(-rel) : std::to_string(rel)) + "_h" + std::to_string(ph);
-                    const std::string acc = "*(const real2*)&P" + std::to_string(ring) + "_" + std::to_string(slot(ring, po)) + "[cb" +
-                                            std::to_string(RR.px) + "_r0 + " + std::to_string(rel) + "]";
-                    // every address the load can form (all pair columns, rows, ring slots) in the rings' SMEM?
-                    const long long cxmin = -PSH, cxmax = 2LL * (CWp - 1) - PSH;
-                    const long long amin = RR.smem_off + (cxmin + rel) * p.es;
-                    const long long amax = RR.smem_off + (long long)(RR.slots - 1) * RR.plane_bytes +
-                                           ((long long)(CH - 1) * RR.px + cxmax + rel + 2) * p.es;
-                    if (L.canvas_ld && amin >= 0 && amax <= L.mbar_off)
-                      o << "      const real2 " << nm << " = " << acc << ";\n";
+                    if (pair_nopred(pk))
+                      o << "      const real2 " << nm << " = " << pair_acc(pk) << ";\n";
                     else
-                      o << "      const real2 " << nm << " = (ca_r0 && cx_r0 >= " << rc[0] << " && cx_r0 < " << rc[1] << " && cy_r0 >= " << rc[2]
-                        << " && cy_r0 < " << rc[3] << ") ? " << acc << " : real2{(real)0, (real)0};\n";
+                      o << "      const real2 " << nm << " = (" << pair_pred(rc) << ") ? " << pair_acc(pk) << " : real2{(real)0, (real)0};\n";
                     it = ldname.emplace(pk, nm).first;
+                    ldfirst_p.emplace(pk, nm);
                   }
                   f = it->second + (comp ? ".y" : ".x");
                   break;
@@ -741,6 +820,15 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
         o << "      }\n";
       }
     }
+    // carried values for the next iteration (ascending plane offset: read before overwritten)
+    for (auto& [pk, src] : pcarry) {
+      std::string val;
+      if (!src.is_load) val = "real2{" + fwd.at(std::make_tuple(src.x, src.v, 0)) + ", " + fwd.at(std::make_tuple(src.x, src.v, 1)) + "}";
+      else if (pcarry.count(src.src)) val = pq_name(src.src);
+      else val = ldfirst_p.at(src.src);
+      o << "      " << pq_name(pk) << " = " << val << ";\n";
+    }
+    if (!pcarry.empty()) o << "      pqv = true;\n";
   };
   auto qname = [](int k, const std::string& ps, int ring, int dz) {
     return "q" + std::to_string(k) + ps + "_" + std::to_string(ring) + "_" + (dz < 0 ? "m" + std::to_string(-dz) : std::to_string(dz));
@@ -1177,6 +1265,7 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
     else emit_canvas();
     o << "    } else {\n";
     if (!carry.empty()) o << "    cqv = false;\n";
+    if (!pcarry.empty()) o << "    pqv = false;\n";
   }
   for (size_t pi = 0; pi < phases.size(); pi++) {
     const auto& ph = phases[pi];
@@ -1218,6 +1307,10 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
         for (int dz = mm.first; dz <= mm.second; dz++)
           o << "  real q" << k << ps << "_" << ring << "_" << (dz < 0 ? "m" + std::to_string(-dz) : std::to_string(dz))
             << " = 0;\n";
+  }
+  if (!pcarry.empty()) {
+    o << "  bool pqv = false;\n";
+    for (auto& [pk, src] : pcarry) o << "  real2 " << pq_name(pk) << " = real2{(real)0, (real)0};\n";
   }
   if (canvas_mode && zq.empty() && !carry.empty()) {
     o << "  bool cqv = false;\n";
