@@ -261,16 +261,18 @@ def cpu_baseline(name: str, budget_s: float = 12.0):
 
 
 # ---------------------------------------------------------------- GPU timing
-AUTOTUNE_CANDIDATES = [  # (tile, stages, zunroll, ringunroll, minblocks, canvas_ld[, pblock x])
+AUTOTUNE_CANDIDATES = [  # (tile, stages, zunroll, ringunroll, minblocks, canvas_ld[, pblock x, pair_zq])
     ((32, 8, 64), 2, 1, 0, 0, 1), ((32, 8, 64), 2, 1, 0, -1, 1), ((32, 8, 64), 2, 1, 0, -1, 0), ((32, 8, 64), 2, 1, 0, 0, 0),
     ((32, 8, 32), 2, 1, 0, -1, 1), ((32, 8, 32), 2, 1, 0, 0, 0), ((32, 8, 0), 2, 1, 0, -1, 1), ((64, 4, 64), 2, 1, 0, 0, 1),
     ((16, 12, 64), 2, 1, 0, 0, 1), ((32, 8, 64), 3, 1, 0, -1, 1), ((32, 8, 64), 2, 1, 1, -1, 1), ((32, 8, 64), 2, 2, 0, 0, 1),
     ((64, 8, 64), 2, 2, 0, 0, 1),   # z-unroll 2 on 64x8: the fastest for the fp32 suite groups (tools/ab.py)
-    # canvas pairs (two x-adjacent points per thread, 16-byte vector shared loads/stores)
-    ((32, 8, 32), 2, 1, 0, -1, 1, 2), ((32, 8, 64), 2, 1, 0, -1, 0, 2), ((32, 8, 64), 2, 1, 0, 0, 1, 2)]
+    # canvas pairs (two x-adjacent points per thread, 16-byte vector shared loads/stores), with and
+    # without z-column register queues
+    ((32, 8, 32), 2, 1, 0, -1, 1, 2, 0), ((32, 8, 64), 2, 1, 0, -1, 1, 2, 0), ((32, 8, 64), 2, 1, 0, -1, 1, 2, 1),
+    ((32, 8, 64), 2, 1, 0, -1, 0, 2, 1), ((32, 8, 64), 2, 1, 0, 0, 1, 2, 1)]
 
 
-def autotune(prog, plan, dev, base_kw, steps=4):
+def autotune(prog, plan, dev, base_kw, steps=6):
     """Per-group launch configuration: run the whole plan under each candidate (tile, stages,
     zunroll) with per-group CUDA-event timing and keep, for every group, its fastest legal
     candidate.  Mutates the arrays (they are synthetic; the timed runs start from the result)."""
@@ -281,8 +283,9 @@ def autotune(prog, plan, dev, base_kw, steps=4):
     for cand in AUTOTUNE_CANDIDATES:
         tile, stages, zu, ru, mb, cl = cand[:6]
         pb = cand[6] if len(cand) > 6 else 1
+        zq = cand[7] if len(cand) > 7 else 1
         kw = dict(base_kw)
-        kw.update(tile=tile, stages=stages, zunroll=zu, ringunroll=ru, minblocks=mb, canvas_ld=cl, pblock=(pb, 1))
+        kw.update(tile=tile, stages=stages, zunroll=zu, ringunroll=ru, minblocks=mb, canvas_ld=cl, pblock=(pb, 1), pair_zq=zq)
         tgt = kf.Target(**kw)
         try:
             ex = kf.Exec(prog, plan, tgt)
@@ -304,7 +307,7 @@ def autotune(prog, plan, dev, base_kw, steps=4):
         del ex, scr
     return ([kf.Target(**kw) for _, kw in best],
             [(list(kw["tile"]), kw["stages"], kw["zunroll"], kw["ringunroll"], kw["minblocks"], kw["canvas_ld"],
-              kw["pblock"][0]) for _, kw in best], tried)
+              kw["pblock"][0], kw["pair_zq"]) for _, kw in best], tried)
 
 
 def max_over_ranks(x: float) -> float:
@@ -430,7 +433,8 @@ def run_kf(args):
         gtargets = [kf.Target(**dict(tkw, tile=tuple(c[0]), stages=c[1], zunroll=c[2], ringunroll=c[3],
                                             minblocks=c[4] if len(c) > 4 else 0,
                                             canvas_ld=c[5] if len(c) > 5 else 1,
-                                            pblock=(c[6] if len(c) > 6 else 1, 1)))
+                                            pblock=(c[6] if len(c) > 6 else 1, 1),
+                                            pair_zq=c[7] if len(c) > 7 else 1))
                     for c in tuned]
     elif args.autotune:
         if rank == 0:
@@ -442,7 +446,8 @@ def run_kf(args):
             gtargets = [kf.Target(**dict(tkw, tile=tuple(c[0]), stages=c[1], zunroll=c[2], ringunroll=c[3],
                                             minblocks=c[4] if len(c) > 4 else 0,
                                             canvas_ld=c[5] if len(c) > 5 else 1,
-                                            pblock=(c[6] if len(c) > 6 else 1, 1)))
+                                            pblock=(c[6] if len(c) > 6 else 1, 1),
+                                            pair_zq=c[7] if len(c) > 7 else 1))
                         for c in tuned]
     rn = Runner(prog, plan, target, gtargets, new_dist_info())
     jit_s = time.time() - t0
@@ -618,7 +623,7 @@ def main():
     ap.add_argument("--autotune", type=int, default=1, help="per-group launch configuration by measurement (1/0)")
     ap.add_argument("--tuned", default=None, help="JSON per-group configs [[tile,stages,zunroll,ringunroll(,minblocks)],...] "
                                                   "(skips autotune; as printed in config.per_group_launch_config: "
-                                                  "[tile, stages, zunroll, ringunroll, minblocks, canvas_ld, pblock_x])")
+                                                  "[tile, stages, zunroll, ringunroll, minblocks, canvas_ld, pblock_x, pair_zq])")
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "kf":
         args.warmup = 3

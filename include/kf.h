@@ -181,8 +181,11 @@ typedef struct {
                                     address they can form lies in the rings' SMEM (fewer
                                     instructions; lanes outside the readers' regions load values
                                     nobody stores), 0 = predicated on the readers' regions      */
+  int32_t pair_zq;               /* pair canvas (pblock 2x1): 1 = z-column values carried in
+                                    registers across stream iterations instead of re-read
+                                    from shared memory (more registers), 0 = off             */
 } kf_target;
-/* Fills the B200 defaults: 8.0e12, 232448, 255, 148, {64,4,0}, 2, 256, 16, 0, 1, {1,1}, 0, 0, 0, 0, 1. */
+/* Fills the B200 defaults: 8.0e12, 232448, 255, 148, {64,4,0}, 2, 256, 16, 0, 1, {1,1}, 0, 0, 0, 0, 1, 1. */
 kf_status kf_target_b200(kf_target* out);
 
 /* ------------------------------------------------------------------ legality (Eq. 1.1-1.7) */

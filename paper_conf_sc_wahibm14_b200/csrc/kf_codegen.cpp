@@ -642,7 +642,7 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
               a = {std::min(a[0], rj[0]), std::max(a[1], rj[1]), std::min(a[2], rj[2]), std::max(a[3], rj[3])};
             }
           }
-    if (!getenv("KF_PAIR_NO_CQ"))   // A/B switch
+    if (L.pair_zq)
       for (auto& [pk, rc] : pall) {
         const auto& [ring, po, rel] = pk;
         const PK nx{ring, po + 1, rel};

@@ -349,6 +349,7 @@ kf_status kf_target_b200(kf_target* out) {
     t.minblocks = 0;
     t.skew = 0;
     t.canvas_ld = 1;
+    t.pair_zq = 1;
     *out = t;
   });
 }

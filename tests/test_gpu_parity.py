@@ -235,7 +235,7 @@ def test_canvas_paths_random_programs(seed, monkeypatch):
 def test_canvas_pairs_random_programs(seed):
     """Pair mode of the canvas (pblock 2x1: two x-adjacent points per thread, 16-byte vector shared
     loads/stores and live-out stores) on random programs with even nx, every boundary condition mix,
-    both dtypes, predicated and unpredicated loads."""
+    both dtypes, predicated and unpredicated loads, with and without z-column register queues."""
     rng = np.random.default_rng(5000 + seed)
     bc = tuple(int(x) for x in rng.integers(0, 2, size=3))
     flags = [0, PROG_RELAX_EXPANDABLE, PROG_RELAX_ALL][seed % 3]
@@ -248,9 +248,9 @@ def test_canvas_pairs_random_programs(seed):
     pick = sorted(legal, key=lambda p: len(set(p)))[:3]
     tile = [(16, 8, 0), (8, 8, 5), (32, 4, 0)][seed % 3]
     for plan in pick:
-        for cl in (0, 1):
-            got, _ = run_kf(desc, plan, inputs, 2, kf.Target(tile=tile, pblock=(2, 1), canvas_ld=cl))
-            assert compare(desc, got, ref) == [], (plan, tile, cl)
+        for cl, zq in ((0, 1), (1, 1), (1, 0)):
+            got, _ = run_kf(desc, plan, inputs, 2, kf.Target(tile=tile, pblock=(2, 1), canvas_ld=cl, pair_zq=zq))
+            assert compare(desc, got, ref) == [], (plan, tile, cl, zq)
 
 
 @pytest.mark.parametrize("cq", [0, 1])
@@ -265,7 +265,8 @@ def test_canvas_weather_knobs(cq, monkeypatch):
     tgt = kf.Target(tile=(32, 8, 0))
     plans = [prog.search(kf.SEARCH_HGGA, tgt, seed=s)[0] for s in (1, 2)]
     for plan in plans:
-        for kw in (dict(), dict(canvas_ld=0), dict(pblock=(2, 1)), dict(pblock=(2, 1), canvas_ld=0), dict(skew=1),
+        for kw in (dict(), dict(canvas_ld=0), dict(pblock=(2, 1)), dict(pblock=(2, 1), canvas_ld=0),
+                   dict(pblock=(2, 1), pair_zq=0), dict(skew=1),
                    dict(minblocks=-1, ringunroll=1), dict(tile=(32, 8, 5))):
             t = kf.Target(**dict(dict(tile=(32, 8, 0)), **kw))
             if kw and prog.validate(plan, t)[0] != 0:   # e.g. V7: skew / ring unrolling need more SMEM

@@ -22,7 +22,8 @@ steps = int(sys.argv[3]) if len(sys.argv) > 3 else 2
 gt = None
 if len(sys.argv) > 4:
     gt = [kf.Target(**dict(kw, tile=tuple(c[0]), stages=c[1], zunroll=c[2], ringunroll=c[3], minblocks=c[4],
-                           canvas_ld=c[5] if len(c) > 5 else 1, pblock=(c[6] if len(c) > 6 else 1, 1)))
+                           canvas_ld=c[5] if len(c) > 5 else 1, pblock=(c[6] if len(c) > 6 else 1, 1),
+                           pair_zq=c[7] if len(c) > 7 else 1))
           for c in json.loads(sys.argv[4])]
 ex = kf.Exec(prog, plan, kf.Target(**kw), group_targets=gt)
 ex.set_graph(False)
