@@ -38,7 +38,7 @@ def main():
     else:
         dev = kf.device_arrays(prog, gen(desc, 3))
     print(json.dumps({"workload": wl, "plan": plan}), flush=True)
-    steps = 10
+    steps = int(os.environ.get("AB_STEPS", "10"))
     for v in variants:
         saved = {}
         for k, val in v.get("env", {}).items():
