@@ -696,6 +696,7 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
       if (ph > 0) o << "      __syncthreads();\n";
       // lanes (first point's canvas x, row) needing each pair load in this phase
       std::map<PK, Rect> prect;
+      std::map<PK, int> pmask;   // elements of the pair needed (bit 0: first, bit 1: second)
       for (int k : cph[ph])
         for (auto& [x, offs] : p.kernels[k].reads)
           for (auto& d : offs)
@@ -705,6 +706,7 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
               const Rect rc = krect.at(load_key(k, x, d, 0));
               const PK pk = pk_of(k, x, d, j, &comp);
               const Rect rj{rc[0] - j, rc[1] - j, rc[2], rc[3]};
+              pmask[pk] |= 1 << comp;
               auto it = prect.find(pk);
               if (it == prect.end()) prect[pk] = rj;
               else {
@@ -712,6 +714,13 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
                 a = {std::min(a[0], rj[0]), std::max(a[1], rj[1]), std::min(a[2], rj[2]), std::max(a[3], rj[3])};
               }
             }
+      // a pair of which only one element is needed (e.g. y/z neighbours in a ring whose pairs are
+      // offset by one from the canvas pairs) is a scalar load: same instruction count as the
+      // vector load, half the wavefronts; carry sources and carried values stay vectors
+      for (auto& [pk, src] : pcarry) {
+        pmask[pk] = 3;
+        if (src.is_load) pmask[src.src] = 3;
+      }
       std::map<PK, std::string> ldname;
       std::vector<std::tuple<int, std::vector<std::string>, std::vector<std::string>>> done;   // (k, vals pt0, vals pt1)
       for (int k : cph[ph]) {
@@ -745,14 +754,24 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
                     const Rect& rc = prect.at(pk);
                     const std::string nm = "pl" + std::to_string(ring) + "_" + (po < 0 ? "m" + std::to_string(-po) : std::to_string(po)) +
                                            "_" + (rel < 0 ? "m" + std::to_string(-rel) : std::to_string(rel)) + "_h" + std::to_string(ph);
-                    if (pair_nopred(pk))
-                      o << "      const real2 " << nm << " = " << pair_acc(pk) << ";\n";
-                    else
-                      o << "      const real2 " << nm << " = (" << pair_pred(rc) << ") ? " << pair_acc(pk) << " : real2{(real)0, (real)0};\n";
+                    const int mask = pmask.at(pk);
+                    if (mask == 3) {
+                      if (pair_nopred(pk))
+                        o << "      const real2 " << nm << " = " << pair_acc(pk) << ";\n";
+                      else
+                        o << "      const real2 " << nm << " = (" << pair_pred(rc) << ") ? " << pair_acc(pk)
+                          << " : real2{(real)0, (real)0};\n";
+                    } else {
+                      const int c1 = mask == 2 ? 1 : 0;
+                      const std::string acc1 = "P" + std::to_string(ring) + "_" + std::to_string(slot(ring, po)) + "[cb" +
+                                               std::to_string(L.rings[ring].px) + "_r0 + " + std::to_string(rel + c1) + "]";
+                      if (pair_nopred(pk)) o << "      const real " << nm << " = " << acc1 << ";\n";
+                      else o << "      const real " << nm << " = (" << pair_pred(rc) << ") ? " << acc1 << " : (real)0;\n";
+                    }
                     it = ldname.emplace(pk, nm).first;
                     ldfirst_p.emplace(pk, nm);
                   }
-                  f = it->second + (comp ? ".y" : ".x");
+                  f = it->second + (pmask.at(pk) == 3 ? (comp ? ".y" : ".x") : "");
                   break;
                 }
                 case KF_OP_NEG: case KF_OP_ABS: case KF_OP_SQRT: {
