@@ -59,7 +59,7 @@ def workload(name: str):
 
 def plan_candidates(prog, target):
     """Candidate plans for measured selection: the paper's search (HGGA) on the projected
-    time with three seeds and on compulsory bytes, greedy merging on projected time, and (weather)
+    time with five seeds (two, plus brute force, for small programs) and on compulsory bytes, greedy merging on projected time, and (weather)
     the App. A.4 hand plan.  Deduplicated by canonical labelling."""
     import paper_conf_sc_wahibm14_b200 as kf
     out, seen = [], set()
@@ -74,8 +74,11 @@ def plan_candidates(prog, target):
     if prog.nk <= 10:
         add(prog.search(kf.SEARCH_BRUTE_TIME, target)[0], "brute-force on projected time")
         add(prog.search(kf.SEARCH_BRUTE, target)[0], "brute-force on compulsory bytes")
+        add(prog.search(kf.SEARCH_GREEDY_TIME, target)[0], "greedy merging on projected time")
+        for seed in (1, 2):
+            add(prog.search(kf.SEARCH_HGGA, target, seed=seed)[0], f"HGGA (seed {seed}) on the resource-aware projected time")
     else:
-        for seed in (1, 2, 3):
+        for seed in (1, 2, 3, 4, 5):
             add(prog.search(kf.SEARCH_HGGA, target, seed=seed)[0], f"HGGA (seed {seed}) on the resource-aware projected time")
         add(prog.search(kf.SEARCH_HGGA_BYTES, target, seed=1)[0], "HGGA (seed 1) on compulsory bytes")
         add(prog.search(kf.SEARCH_GREEDY_TIME, target)[0], "greedy merging on projected time")
