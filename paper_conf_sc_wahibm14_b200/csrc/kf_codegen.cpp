@@ -692,12 +692,24 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
       }
       o << "      }\n";
     }
+    // Loads are shared across the phases of an iteration: a (ring, plane, offset) value cannot
+    // change within an iteration (a reader of a version follows its producer's phase; ring depths
+    // keep recycled slots dead), and pair mode has the registers to keep them (one point per
+    // thread reloads after every barrier instead).  KF_PAIR_PHASE_LD=1: per-phase loads (A/B).
+    const bool phase_ld = getenv("KF_PAIR_PHASE_LD") != nullptr;
+    std::map<PK, Rect> prect;
+    std::map<PK, int> pmask;   // elements of the pair needed (bit 0: first, bit 1: second)
+    std::map<PK, std::string> ldname;
     for (size_t ph = 0; ph < cph.size(); ph++) {
       if (ph > 0) o << "      __syncthreads();\n";
-      // lanes (first point's canvas x, row) needing each pair load in this phase
-      std::map<PK, Rect> prect;
-      std::map<PK, int> pmask;   // elements of the pair needed (bit 0: first, bit 1: second)
-      for (int k : cph[ph])
+      // lanes (first point's canvas x, row) needing each pair load in this phase (all phases
+      // unless per-phase loads)
+      if (phase_ld || ph == 0) {
+        prect.clear();
+        pmask.clear();
+        ldname.clear();
+      }
+      for (int k : (phase_ld ? cph[ph] : ph == 0 ? alive : std::vector<int>{}))
         for (auto& [x, offs] : p.kernels[k].reads)
           for (auto& d : offs)
             for (int j = 0; j < 2; j++) {
@@ -721,7 +733,6 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
         pmask[pk] = 3;
         if (src.is_load) pmask[src.src] = 3;
       }
-      std::map<PK, std::string> ldname;
       std::vector<std::tuple<int, std::vector<std::string>, std::vector<std::string>>> done;   // (k, vals pt0, vals pt1)
       for (int k : cph[ph]) {
         const Kernel& K = p.kernels[k];
