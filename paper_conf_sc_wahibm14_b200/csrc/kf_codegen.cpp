@@ -445,8 +445,10 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
     std::map<std::pair<Key, int>, std::string> ldfirst;   // first load of every key (carry sources)
     for (size_t ph = 0; ph < cph.size(); ph++) {
       if (ph > 0) o << "      __syncthreads();\n";
-      // loads are shared within a phase only: values do not stay live across barriers (registers)
-      ldname.clear();
+      // loads are shared across the phases of an iteration (a value cannot change within an
+      // iteration; measured 1-5 % faster on the flux groups despite the longer live ranges);
+      // KF_CANVAS_PHASE_LD=1: per-phase loads (A/B)
+      if (getenv("KF_CANVAS_PHASE_LD")) ldname.clear();
       std::vector<std::tuple<int, int, int, std::vector<std::string>>> done;   // (k, r, uu, vals)
       for (int k : cph[ph]) {
         const Kernel& K = p.kernels[k];
