@@ -439,6 +439,10 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
     return std::string(pre) + std::to_string(key.ring) + "_" + (key.po < 0 ? "m" + std::to_string(-key.po) : std::to_string(key.po)) +
            "_" + (key.off < 0 ? "m" + std::to_string(-key.off) : std::to_string(key.off)) + rs;
   };
+  // shared loads reused across the phases of an iteration: a value cannot change within an
+  // iteration, but the longer live ranges cost registers -- large groups (a 35-kernel group
+  // spilled) keep per-phase loads.  KF_CANVAS_PHASE_LD=1: per-phase loads everywhere (A/B).
+  const bool xphase_ld = alive.size() <= 16 && cv.phases.size() <= 4 && !getenv("KF_CANVAS_PHASE_LD");
   auto emit_canvas = [&]() {
     std::map<std::pair<Key, int>, std::string> ldname;
     std::map<std::tuple<int, int, int, int>, std::string> fwd;   // (x, v, round, sub-plane) -> value
@@ -448,7 +452,7 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
       // loads are shared across the phases of an iteration (a value cannot change within an
       // iteration; measured 1-5 % faster on the flux groups despite the longer live ranges);
       // KF_CANVAS_PHASE_LD=1: per-phase loads (A/B)
-      if (getenv("KF_CANVAS_PHASE_LD")) ldname.clear();
+      if (!xphase_ld) ldname.clear();
       std::vector<std::tuple<int, int, int, std::vector<std::string>>> done;   // (k, r, uu, vals)
       for (int k : cph[ph]) {
         const Kernel& K = p.kernels[k];
@@ -697,8 +701,8 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
     // Loads are shared across the phases of an iteration: a (ring, plane, offset) value cannot
     // change within an iteration (a reader of a version follows its producer's phase; ring depths
     // keep recycled slots dead), and pair mode has the registers to keep them (one point per
-    // thread reloads after every barrier instead).  KF_PAIR_PHASE_LD=1: per-phase loads (A/B).
-    const bool phase_ld = getenv("KF_PAIR_PHASE_LD") != nullptr;
+    // thread reloads after every barrier instead; xphase_ld above).
+    const bool phase_ld = !xphase_ld;
     std::map<PK, Rect> prect;
     std::map<PK, int> pmask;   // elements of the pair needed (bit 0: first, bit 1: second)
     std::map<PK, std::string> ldname;
