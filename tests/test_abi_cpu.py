@@ -232,3 +232,26 @@ def test_paper_projection_abi_matches_oracle_and_example():
     assert out.p_membound_gflops == ref["p_membound_gflops"]
     assert out.t_pro_s == ref["t_pro_s"]
     assert out.eq2_ok and out.eq3_ok is not None
+
+
+def test_target_knobs_validated():
+    """kf_target launch knobs outside their ranges are KF_E_ARG (no silent clamping)."""
+    desc = P.tiny()
+    p = kf.Program(desc)
+    for bad in (dict(canvas_ld=2), dict(pair_zq=-1), dict(skew=2), dict(minblocks=-2), dict(pblock=(5, 1)),
+                dict(tile=(30, 8, 0))):
+        with pytest.raises(kf.KfError):
+            p.project([0, 0, 1], kf.Target(**bad))
+
+
+def test_codegen_pair_canvas_and_split_compile_for_sm100a():
+    """The pair canvas (pblock 2x1: vector shared loads/stores, z register queues) and the
+    interior/boundary unit split compile for sm_100a without spills on the weather groups."""
+    desc = P.weather(n=(64, 48, 12))
+    p = kf.Program(desc)
+    t = kf.Target(tile=(32, 8, 0))
+    plan, _ = p.search(kf.SEARCH_HGGA, t, seed=2)
+    for g in range(max(plan) + 1):
+        for kw in (dict(pblock=(2, 1)), dict(pblock=(2, 1), canvas_ld=0, pair_zq=0)):
+            regs, spill, log = p.jit_check(plan, g, kf.Target(tile=(32, 8, 0), **kw))
+            assert "sm_100a" in log and spill == 0, (g, kw, spill)
