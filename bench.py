@@ -273,7 +273,7 @@ AUTOTUNE_CANDIDATES = [  # (tile, stages, zunroll, ringunroll, minblocks, canvas
     # canvas pairs (two x-adjacent points per thread, 16-byte vector shared loads/stores), with and
     # without z-column register queues
     ((32, 8, 32), 2, 1, 0, -1, 1, 2, 0), ((32, 8, 64), 2, 1, 0, -1, 1, 2, 0), ((32, 8, 64), 2, 1, 0, -1, 1, 2, 1),
-    ((32, 8, 64), 2, 1, 0, -1, 0, 2, 1), ((32, 8, 64), 2, 1, 0, 0, 1, 2, 1)]
+    ((32, 8, 64), 2, 1, 0, -1, 0, 2, 1), ((32, 8, 64), 2, 1, 0, 0, 1, 2, 1), ((32, 8, 32), 2, 1, 0, -1, 1, 2, 1)]
 
 
 def autotune(prog, plan, dev, base_kw, steps=6):
