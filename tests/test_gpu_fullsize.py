@@ -71,3 +71,40 @@ def test_weather_full_size_sampled_windows():
             ys = (np.arange(y0, y0 + w) % 512) + g[1]
             gv = got[nm][g[2]:g[2] + 128][:, ys][:, :, xs]
             assert np.array_equal(bits(gv), bits(r)), (nm, x0, y0)
+
+
+def test_weather_full_size_bench_configuration():
+    """The exact configuration of the committed bench line (profiles/round1_s3_bench_final.json:
+    its plan labels and autotuned per-group launch configurations -- canvas pairs, z register
+    queues, unpredicated loads, TMA stages, z chunks), at full size, on sampled windows."""
+    import json
+    import os
+    line = json.load(open(os.path.join(os.path.dirname(__file__), "..", "profiles", "round1_s3_bench_final.json")))
+    plan = line["config"]["plan_labels"]
+    tuned = line["config"]["per_group_launch_config"]
+    desc = P.weather(n=(512, 512, 128))
+    inputs = D.weather_inputs(desc, 3)
+    prog = kf.Program(desc)
+    gt = [kf.Target(tile=tuple(c[0]), stages=c[1], zunroll=c[2], ringunroll=c[3], minblocks=c[4], canvas_ld=c[5],
+                    pblock=(c[6], 1), pair_zq=c[7]) for c in tuned]
+    nsteps = 2
+    ex = kf.Exec(prog, plan, kf.Target(tile=(32, 8, 64)), group_targets=gt)
+    dev = kf.device_arrays(prog, inputs)
+    sb = ex.scratch_bytes()
+    scr = torch.empty(sb, dtype=torch.uint8, device="cuda") if sb else None
+    ex.run(dev, scr, nsteps)
+    torch.cuda.synchronize()
+    got = kf.host_arrays(prog, dev)
+    del dev, scr
+    M = dependency_radius(desc, nsteps) + 1
+    w = 8
+    g = desc.ghost
+    for (x0, y0) in ((0, 0), (508, 3), (200, 505), (131, 257), (64, 64)):
+        sub, sin = crop(desc, inputs, x0, y0, w, M)
+        ref = interp.run(sub, sin, nsteps)
+        for nm in ("DENS", "MOMX", "MOMY", "MOMZ", "RHOT"):
+            r = ref[nm][g[2]:g[2] + 128, g[1] + M:g[1] + M + w, g[0] + M:g[0] + M + w]
+            xs = (np.arange(x0, x0 + w) % 512) + g[0]
+            ys = (np.arange(y0, y0 + w) % 512) + g[1]
+            gv = got[nm][g[2]:g[2] + 128][:, ys][:, :, xs]
+            assert np.array_equal(bits(gv), bits(r)), (nm, x0, y0)
