@@ -158,5 +158,6 @@ def test_loopback_overlap_interior_boundary_split(overlap):
     tgt = kf.Target(tile=(16, 8, 0))
     plans = [P.weather_hand_plan(desc), kf.Program(desc).search(kf.SEARCH_HGGA, tgt, seed=1)[0]]
     for plan in plans:
-        got = _run_loopback(desc, plan, inputs, 3, 2, 2, tgt, overlap=overlap)
-        assert compare(desc, got, ref) == [], (overlap, plan)
+        for t in (tgt, kf.Target(tile=(16, 8, 0), pblock=(2, 1))):   # single points and canvas pairs
+            got = _run_loopback(desc, plan, inputs, 3, 2, 2, t, overlap=overlap)
+            assert compare(desc, got, ref) == [], (overlap, plan, t.pblock)
