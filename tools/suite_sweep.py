@@ -3,7 +3,8 @@
 For every (kernels, arrays) pair the suite generator (workloads.programs.gen_suite)
 builds a program with average thread load `--load` (Table V: 4..12; Fig. 9 uses 8).  Each program
 runs unfused (singleton groups) and under the plans the searches propose (HGGA on the projected time
-and on compulsory bytes); every plan is timed with CUDA events after warm-up.  One JSON
+and on compulsory bytes); every plan is timed with CUDA events after warm-up, with single
+canvas points and with canvas pairs (the faster is kept, for the unfused baseline too).  One JSON
 line per benchmark: speedup of the fastest fused plan over unfused, Fusion Efficiency (Eq. 12,
 P:501), projected vs measured time, compulsory bytes.
 
@@ -48,7 +49,23 @@ def main():
     import paper_conf_sc_wahibm14_b200 as kf
     from workloads import programs as P
     n = tuple(int(v) for v in args.n.split(","))
-    target = kf.Target(tile=(32, 8, 64))
+    # launch configurations tried for every plan (the fastest is kept): single canvas points and
+    # canvas pairs (two x-adjacent points per thread, vector shared loads)
+    targets = [kf.Target(tile=(32, 8, 64)), kf.Target(tile=(32, 8, 64), pblock=(2, 1))]
+    target = targets[0]
+
+    def best_time(prog, plan, dev):
+        best = None
+        for t in targets:
+            try:
+                r = time_plan(kf, prog, plan, dev, t, args.steps)
+            except Exception:   # noqa: BLE001 -- a configuration illegal for this plan (V7/V8)
+                continue
+            if best is None or r[0] < best[0]:
+                best = r
+        if best is None:
+            raise RuntimeError("no legal launch configuration")
+        return best
     for nk in [int(v) for v in args.kernels.split(",")]:
         for na in [int(float(r) * nk) for r in args.ratios.split(",")]:
             t0 = time.time()
@@ -61,13 +78,13 @@ def main():
             L = prog.layout()
             g = torch.Generator(device="cuda").manual_seed(args.seed)
             dev = [torch.rand(L.elems, generator=g, device="cuda", dtype=torch.float32) * 2 - 1 for _ in desc.arrays]
-            ms_u, b_u, _ = time_plan(kf, prog, list(range(nk)), dev, target, args.steps)
+            ms_u, b_u, _ = best_time(prog, list(range(nk)), dev)
             res = []
             for name, method in (("hgga_time", kf.SEARCH_HGGA), ("hgga_bytes", kf.SEARCH_HGGA_BYTES)):
                 plan, _ = prog.search(method, target, seed=1)
                 per, _, t_proj = prog.project(plan, target)
                 try:
-                    ms, b, m = time_plan(kf, prog, plan, dev, target, args.steps)
+                    ms, b, m = best_time(prog, plan, dev)
                 except Exception as e:   # noqa: BLE001 -- report and continue the sweep
                     res.append({"plan": name, "error": str(e)[:160]})
                     continue
