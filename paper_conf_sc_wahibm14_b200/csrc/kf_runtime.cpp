@@ -76,6 +76,7 @@ struct Compiled {
   std::vector<char> cubin;
   std::string log;
   int regs_ptxas = -1, spill = -1;
+  bool nocap = false;   // compiled with KF_NO_MAXNREG (register cap dropped)
 };
 
 static Compiled nvrtc_compile(const std::string& src, const std::string& name) {
@@ -103,7 +104,8 @@ static Compiled nvrtc_compile(const std::string& src, const std::string& name) {
   nvrtcGetCUBIN(prog, c.cubin.data());
   nvrtcDestroyProgram(&prog);
   if (const char* dir = getenv("KF_DUMP_DIR")) {   // debugging aid: keep the generated source and cubin
-    std::string base = std::string(dir) + "/" + name;
+    std::string base = std::string(dir) + "/" + name + (src.rfind("#define KF_NO_MAXNREG", 0) == 0 ? "_nomaxnreg" : "");
+    if (FILE* f = fopen((base + ".log").c_str(), "w")) { fwrite(c.log.data(), 1, c.log.size(), f); fclose(f); }
     if (FILE* f = fopen((base + ".cu").c_str(), "w")) { fwrite(src.data(), 1, src.size(), f); fclose(f); }
     if (FILE* f = fopen((base + ".cubin").c_str(), "wb")) { fwrite(c.cubin.data(), 1, c.cubin.size(), f); fclose(f); }
   }
@@ -129,8 +131,21 @@ static std::shared_ptr<Compiled> compile_cached(const std::string& src, const st
   }
   auto c = std::make_shared<Compiled>(nvrtc_compile(src, name));
   // the register cap (__maxnreg__, occupancy) must not cost local-memory spills
-  if (c->spill > 0 && src.find("__maxnreg__") != std::string::npos)
+  if (c->spill > 0 && src.find("__maxnreg__") != std::string::npos) {
     c = std::make_shared<Compiled>(nvrtc_compile("#define KF_NO_MAXNREG 1\n" + src, name));
+    c->nocap = true;
+  }
+  std::lock_guard<std::mutex> lk(g_cache_mu);
+  g_cubin_cache[src] = c;
+  return c;
+}
+
+// The ptxas statistics come from the NVRTC log, which is empty when NVRTC serves a program from
+// its own on-disk cache (seen on reused GPU boxes): the spill test above then never fires.  The
+// loader checks the function's local memory instead and comes here for the uncapped build.
+static std::shared_ptr<Compiled> compile_nocap(const std::string& src, const std::string& name) {
+  auto c = std::make_shared<Compiled>(nvrtc_compile("#define KF_NO_MAXNREG 1\n" + src, name));
+  c->nocap = true;
   std::lock_guard<std::mutex> lk(g_cache_mu);
   g_cubin_cache[src] = c;
   return c;
@@ -377,12 +392,19 @@ static void ensure_device(kf_exec* E) {
   E->device = dev;
   const Program& p = E->prog->p;
   for (auto& g : E->G) {
-    ckd(drv().moduleLoadData(&g.mod, g.comp->cubin.data()), ("cuModuleLoadData " + g.cg.name).c_str());
-    ckd(drv().moduleGetFunction(&g.fn, g.mod, g.cg.name.c_str()), "cuModuleGetFunction");
-    ckd(drv().funcSetAttribute(g.fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, g.smem),
-        "cuFuncSetAttribute(MAX_DYNAMIC_SHARED_SIZE_BYTES)");
-    drv().funcGetAttribute(&g.regs, CU_FUNC_ATTRIBUTE_NUM_REGS, g.fn);
-    drv().funcGetAttribute(&g.local, CU_FUNC_ATTRIBUTE_LOCAL_SIZE_BYTES, g.fn);
+    for (int attempt = 0; attempt < 2; attempt++) {
+      ckd(drv().moduleLoadData(&g.mod, g.comp->cubin.data()), ("cuModuleLoadData " + g.cg.name).c_str());
+      ckd(drv().moduleGetFunction(&g.fn, g.mod, g.cg.name.c_str()), "cuModuleGetFunction");
+      ckd(drv().funcSetAttribute(g.fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, g.smem),
+          "cuFuncSetAttribute(MAX_DYNAMIC_SHARED_SIZE_BYTES)");
+      drv().funcGetAttribute(&g.regs, CU_FUNC_ATTRIBUTE_NUM_REGS, g.fn);
+      drv().funcGetAttribute(&g.local, CU_FUNC_ATTRIBUTE_LOCAL_SIZE_BYTES, g.fn);
+      // the register cap must not cost local memory (spills): rebuild without it
+      if (g.local > 0 && !g.comp->nocap && g.cg.source.find("__maxnreg__") != std::string::npos)
+        g.comp = compile_nocap(g.cg.source, g.cg.name);
+      else
+        break;
+    }
   }
   (void)p;
 }
