@@ -2,23 +2,32 @@
 """Benchmark of the fused stencil-program hot path on B200 (BASELINE.json metric).
 
 One *step* = one pass of the whole hot path over the program: every fused group of the
-plan (plus periodic ghost fills) in quotient-topological order = one timestep of the
-44-kernel / 31-array weather-shaped program (BASELINE config 3, 512x512x128 fp64).
+plan in quotient-topological order (periodic ghosts written by the producing groups; halo
+exchanges between ranks at N > 1) = one timestep of the 44-kernel / 31-array weather-shaped
+program (BASELINE config 3, 512x512x128 fp64 per GPU).
 
 Printed JSON (rank 0, one line): metric/value = grid-points*steps/s of the fused plan with
-inputs resident in HBM (CUDA events on the launch stream, max over ranks), plus the
-roofline of the dominant group kernel, the oracle's CPU baseline, the end-to-end number
-through kf_run_host (host buffers, copies inside the timed region), the unfused plan's
-speed (speedup vs unfused), the projection, Fusion Efficiency (Eq. 12) and SM clocks.
+inputs resident in HBM (CUDA events on the launch stream, max over ranks), plus the roofline of
+the dominant group kernel, per-group measured vs projected times (NEXT-2), the parity of the
+timed configuration on sampled windows against the oracle, the oracle's CPU baseline (1 core and
+all cores), the end-to-end number through kf_run_host (host buffers, copies inside the timed
+region), the unfused plan's speed (speedup vs unfused), Fusion Efficiency (Eq. 12) and SM clocks.
 
-  python bench.py [--gpus N --steps K --warmup W] [--workload weather|tiny|fig3|stress]
-  python bench.py --impl reference ...     # the oracle on host cores, same metric/config
+  python bench.py [--gpus N --steps K --warmup W] [--workload weather|weak|stress|suite|tiny]
+  python bench.py --workload suite --all-plans        # config 2: every legal plan timed
+  python bench.py --impl reference ...                # the oracle on host cores, same metric/config
+
+--gpus N > 1 without a launcher re-executes itself under torch.distributed.run (one rank per
+GPU); with a launcher WORLD_SIZE must equal N.  Workloads: weather = config 3 (weak scaling,
+512x512x128 per GPU), weak = config 4 (1024x1024x128 per GPU), stress = config 5 (768^3 global,
+strong scaling over a px x py split), suite = config 2 (256^3 fp32), tiny = config 1.
 """
 from __future__ import annotations
 
 import argparse
 import json
 import os
+import socket
 import subprocess
 import sys
 import threading
@@ -32,35 +41,121 @@ METRIC = "fused-program grid-pts·steps/s"
 UNIT = "grid-pts·steps/s"
 
 
+def grid_for(world):
+    return {1: (1, 1), 2: (2, 1), 4: (2, 2), 8: (4, 2)}.get(world, (world, 1))
+
+
 # ---------------------------------------------------------------- workloads
-def workload(name: str):
-    """(program description, input generator, target kwargs, label)."""
-    from workloads import data, programs
-    if name == "weather":
-        desc = programs.weather(n=(512, 512, 128))
-        return desc, data.weather_inputs, dict(tile=(32, 8, 64)), "weather-44k31a-512x512x128-fp64 (BASELINE config 3)"
-    if name == "weather_small":
-        desc = programs.weather(n=(128, 128, 64))
-        return desc, data.weather_inputs, dict(tile=(32, 16, 0)), "weather-44k31a-128x128x64-fp64"
-    if name == "suite":
-        desc = programs.gen_suite(seed=0)
-        return desc, data.uniform, dict(tile=(32, 8, 0)), "suite-10k8a-256^3-fp32 (BASELINE config 2, gen_suite seed 0)"
-    if name == "tiny":
-        desc = programs.tiny()
-        return desc, data.uniform, dict(tile=(32, 16, 0)), "tiny-3k3a-32^3-fp32 (BASELINE config 1)"
-    if name == "fig3":
-        desc = programs.fig3(n=(512, 512, 128))
-        return desc, data.fig3_inputs, dict(tile=(32, 16, 0)), "fig3-6k-512x512x128-fp64"
-    if name == "stress":
-        desc = programs.stress(m=2, n=(768, 768, 768))
-        return desc, None, dict(tile=(32, 8, 0), max_halo=16), "stress-2fields-L25xL25-768^3-fp64 (config 5)"
-    raise SystemExit(f"unknown workload {name}")
+class Workload:
+    """The per-rank (local) program, its input generator and labels.  `global_n` is the grid the
+    whole job covers (weak: per-GPU grid x ranks; strong: fixed)."""
+
+    def __init__(self, name: str, world: int):
+        from workloads import programs
+        self.name = name
+        px, py = grid_for(world)
+        self.scaling = "weak"
+        self.tile_grid = None
+        if name == "weather":
+            self.desc = programs.weather(n=(512, 512, 128))
+            self.gen = "weather"
+            self.tkw = dict(tile=(32, 8, 64))
+            self.label = "weather-44k31a-512x512x128-fp64 per GPU (BASELINE config 3)"
+        elif name == "weak":
+            # config 4: 1024x1024x128 per GPU; fields generated at 512x512x128 and tiled 2x2 on the device
+            self.desc = programs.weather(n=(1024, 1024, 128))
+            self.gen = "weather_tiled"
+            self.tile_grid = (512, 512, 128)
+            self.tkw = dict(tile=(32, 8, 64))
+            self.label = "weather-44k31a-1024x1024x128-fp64 per GPU (BASELINE config 4, weak)"
+        elif name == "weather_small":
+            self.desc = programs.weather(n=(128, 128, 64))
+            self.gen = "weather"
+            self.tkw = dict(tile=(32, 16, 0))
+            self.label = "weather-44k31a-128x128x64-fp64"
+        elif name == "suite":
+            self.desc = programs.gen_suite(seed=0)
+            self.gen = "uniform"
+            self.tkw = dict(tile=(32, 8, 0))
+            self.label = "suite-10k8a-256^3-fp32 (BASELINE config 2, gen_suite seed 0)"
+        elif name == "tiny":
+            self.desc = programs.tiny()
+            self.gen = "uniform"
+            self.tkw = dict(tile=(32, 16, 0))
+            self.label = "tiny-3k3a-32^3-fp32 (BASELINE config 1)"
+        elif name == "fig3":
+            self.desc = programs.fig3(n=(512, 512, 128))
+            self.gen = "fig3"
+            self.tkw = dict(tile=(32, 16, 0))
+            self.label = "fig3-6k-512x512x128-fp64"
+        elif name == "stress":
+            # config 5: 768^3 global, strong scaling over the px x py process grid
+            if 768 % px or 768 % py:
+                raise SystemExit(f"stress: 768 not divisible by the process grid {px}x{py}")
+            self.desc = programs.stress(m=2, n=(768 // px, 768 // py, 768))
+            self.gen = "device_uniform"
+            self.tkw = dict(tile=(32, 8, 0), max_halo=16)
+            self.scaling = "strong"
+            self.label = f"stress-2fields-L25xL25-768^3-fp64 (config 5, strong; local {768 // px}x{768 // py}x768)"
+        else:
+            raise SystemExit(f"unknown workload {name}")
+        self.world = world
+        # weak: every rank owns a full per-GPU grid; strong: the local grids partition the global one
+        self.global_npts = self.desc.npts * world
+
+    def inputs(self, prog, rank, device_ok=True):
+        """Device tensors (kf layout) of the rank's seeded synthetic inputs."""
+        import torch
+        import paper_conf_sc_wahibm14_b200 as kf
+        from workloads import data, programs
+        seed = 3 + rank
+        if self.gen == "device_uniform":
+            L = prog.layout()
+            gdev = torch.Generator(device="cuda").manual_seed(seed)
+            dt = torch.float64 if self.desc.dtype == 1 else torch.float32
+            return [torch.rand(L.elems, generator=gdev, device="cuda", dtype=dt) * 2 - 1 for _ in self.desc.arrays], None
+        if self.gen == "weather_tiled":
+            small = programs.weather(n=self.tile_grid)
+            sin = data.weather_inputs(small, seed)
+            return tile_to_device(prog, small, sin), None
+        if self.gen == "weather":
+            inp = data.weather_inputs(self.desc, seed)
+        elif self.gen == "fig3":
+            inp = data.fig3_inputs(self.desc, seed)
+        else:
+            inp = data.uniform(self.desc, seed)
+        return kf.device_arrays(prog, inp), inp
+
+
+def tile_to_device(prog, small, sin):
+    """Periodic xy tiling of a small field set into the program's (larger) grid, on the device:
+    interior (k, j, i) <- small interior (k, j mod ny_s, i mod nx_s); x/y ghosts wrap; z ghosts are
+    the small grid's (plumbing: synthetic inputs only)."""
+    import torch
+    d = prog.desc
+    L = prog.layout()
+    g = d.ghost
+    nxs, nys, nzs = small.n
+    assert nzs == d.n[2] and small.ghost == d.ghost
+    xi = torch.tensor([(i % nxs) + g[0] for i in range(-g[0], d.n[0] + g[0])], device="cuda")
+    yi = torch.tensor([(j % nys) + g[1] for j in range(-g[1], d.n[1] + g[1])], device="cuda")
+    out = []
+    for nm, _ in d.arrays:
+        s = torch.from_numpy(sin[nm]).to("cuda")
+        big = s[:, yi][:, :, xi]
+        flat = torch.zeros(L.elems, dtype=s.dtype, device="cuda")
+        v = flat.view(d.n[2] + 2 * g[2], L.rows, L.pitch)
+        v[:, :, L.xoff - g[0]:L.xoff + d.n[0] + g[0]] = big
+        out.append(flat)
+        del s, big
+    return out
 
 
 def plan_candidates(prog, target):
     """Candidate plans for measured selection: the paper's search (HGGA) on the projected
-    time with five seeds (two, plus brute force, for small programs) and on compulsory bytes, greedy merging on projected time, and (weather)
-    the App. A.4 hand plan.  Deduplicated by canonical labelling."""
+    time with five seeds (two, plus brute force, for small programs) and on compulsory bytes, greedy
+    merging on projected time, and (weather) the App. A.4 hand plan.  Deduplicated by canonical
+    labelling."""
     import paper_conf_sc_wahibm14_b200 as kf
     out, seen = [], set()
 
@@ -88,12 +183,25 @@ def plan_candidates(prog, target):
     return out
 
 
+def time_exec(ex, dev, steps, warm=2):
+    import torch
+    sb = ex.scratch_bytes()
+    scr = torch.empty(sb, dtype=torch.uint8, device="cuda") if sb else None
+    ex.run(dev, scr, warm)
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    ex.run(dev, scr, steps)
+    e1.record()
+    torch.cuda.synchronize()
+    return e0.elapsed_time(e1) / steps
+
+
 def select_plan(prog, target, dev, steps=5):
     """Measured selection among plan_candidates(): every candidate is compiled with the default
     launch configuration and timed (CUDA events, `steps` steps after 2 warm-up steps); the
     fastest is kept.  The projection ranks plans inside the search; the measurement decides
     between the few it proposes."""
-    import torch
     import paper_conf_sc_wahibm14_b200 as kf
     res = []
     for plan, kind in plan_candidates(prog, target):
@@ -102,17 +210,8 @@ def select_plan(prog, target, dev, steps=5):
         except Exception as e:   # an illegal candidate for this target: skip it
             res.append((float("inf"), plan, kind + f" (failed: {str(e)[:80]})"))
             continue
-        sb = ex.scratch_bytes()
-        scr = torch.empty(sb, dtype=torch.uint8, device="cuda") if sb else None
-        ex.run(dev, scr, 2)
-        torch.cuda.synchronize()
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record()
-        ex.run(dev, scr, steps)
-        e1.record()
-        torch.cuda.synchronize()
-        res.append((e0.elapsed_time(e1) / steps, plan, kind))
-        del ex, scr
+        res.append((time_exec(ex, dev, steps), plan, kind))
+        del ex
     best = min(res, key=lambda r: r[0])
     ranked = [(plan, kind) for ms, plan, kind in sorted(res, key=lambda r: r[0]) if ms < float("inf")]
     return best[1], best[2] + " (fastest of the measured candidates)", [
@@ -232,26 +331,28 @@ def ncu_traffic(kernel_name: str):
 
 
 # ---------------------------------------------------------------- CPU baseline (oracle)
-def cpu_baseline(name: str, budget_s: float = 12.0):
-    """The oracle (numpy, 1 thread) on a bounded sample of the same workload."""
-    from oracle import interp
+def _oracle_sample(name: str):
     from workloads import programs, data
-    if name.startswith("weather"):
-        desc = programs.weather(n=(96, 96, 128))
-        inp = data.weather_inputs(desc, 3)
-        sample = "weather program on a 96x96x128 sub-grid, 1 step per timing (numpy oracle, unfused)"
-    elif name == "tiny":
+    if name in ("weather", "weak", "weather_small"):
+        desc = programs.weather(n=(64, 64, 128))
+        return desc, data.weather_inputs(desc, 3), "weather program on a 64x64x128 sub-grid"
+    if name == "tiny":
         desc = programs.tiny()
-        inp = data.uniform(desc, 1)
-        sample = "tiny 32^3, 1 step per timing"
-    elif name == "fig3":
-        desc = programs.fig3(n=(128, 128, 128))
-        inp = data.fig3_inputs(desc, 3)
-        sample = "fig3 on 128^3, 1 step"
-    else:
-        desc = programs.stress(m=2, n=(96, 96, 96))
-        inp = data.uniform(desc, 5)
-        sample = "stress 2 fields on 96^3, 1 step"
+        return desc, data.uniform(desc, 1), "tiny 32^3"
+    if name == "fig3":
+        desc = programs.fig3(n=(64, 64, 128))
+        return desc, data.fig3_inputs(desc, 3), "fig3 on 64x64x128"
+    if name == "suite":
+        desc = programs.gen_suite(seed=0, n=(64, 64, 64))
+        return desc, data.uniform(desc, 3), "suite program on 64^3"
+    desc = programs.stress(m=2, n=(64, 64, 64))
+    return desc, data.uniform(desc, 5), "stress 2 fields on 64^3"
+
+
+def _oracle_worker(args):
+    name, budget_s = args
+    from oracle import interp
+    desc, inp, _ = _oracle_sample(name)
     t0 = time.perf_counter()
     steps = 0
     while True:
@@ -259,9 +360,41 @@ def cpu_baseline(name: str, budget_s: float = 12.0):
         steps += 1
         if time.perf_counter() - t0 > budget_s:
             break
-    dt = time.perf_counter() - t0
-    return {"value": desc.npts * steps / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
-            "sample": f"{sample}; {steps} step(s) in {dt:.1f} s"}
+    return desc.npts * steps, time.perf_counter() - t0
+
+
+def cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return "unknown"
+
+
+def cpu_baseline(name: str, budget_s: float = 8.0):
+    """The oracle (numpy, unfused, as it stands) on bounded samples of the same workload: one
+    process on one core, then one process per host core (each on its own sub-grid, capped at 64)."""
+    import multiprocessing as mp
+    pts, dt = _oracle_worker((name, budget_s))
+    _, _, sample = _oracle_sample(name)
+    one = pts / dt
+    ncores = min(os.cpu_count() or 1, 64)
+    allc = None
+    if ncores > 1:
+        try:
+            ctx = mp.get_context("fork")
+            t0 = time.perf_counter()
+            with ctx.Pool(ncores) as pool:
+                res = pool.map(_oracle_worker, [(name, budget_s)] * ncores)
+            wall = time.perf_counter() - t0
+            allc = {"value": sum(r[0] for r in res) / wall, "cores": ncores, "wall_s": round(wall, 2)}
+        except Exception as e:   # reported, never guessed
+            allc = {"error": f"{type(e).__name__}: {e}"}
+    return {"value": one, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"{sample}, numpy oracle unfused, 1 step per timing, {budget_s:.0f} s budget per process",
+            "all_cores": allc, "host_cpu": cpu_model(), "host_cores": os.cpu_count()}
 
 
 # ---------------------------------------------------------------- GPU timing
@@ -279,23 +412,33 @@ AUTOTUNE_CANDIDATES = [  # (tile, stages, zunroll, ringunroll, minblocks, canvas
     ((32, 8, 43), 2, 1, 0, -1, 1, 2, 1), ((32, 8, 43), 2, 1, 0, -1, 1, 2, 0), ((32, 8, 43), 2, 1, 0, -1, 1)]
 
 
+def cand_kw(base_kw, c):
+    kw = dict(base_kw)
+    kw.update(tile=tuple(c[0]), stages=c[1], zunroll=c[2], ringunroll=c[3], minblocks=c[4] if len(c) > 4 else 0,
+              canvas_ld=c[5] if len(c) > 5 else 1, pblock=(c[6] if len(c) > 6 else 1, 1),
+              pair_zq=c[7] if len(c) > 7 else 1)
+    return kw
+
+
+def cand_norm(c):
+    """Full 8-field form [tile, stages, zunroll, ringunroll, minblocks, canvas_ld, pblock_x, pair_zq]."""
+    full = list(c) + [None] * (8 - len(c))
+    dflt = [None, 2, 1, 0, 0, 1, 1, 1]
+    return [list(full[0])] + [full[i] if full[i] is not None else dflt[i] for i in range(1, 8)]
+
+
 def autotune(prog, plan, dev, base_kw, steps=6):
     """Per-group launch configuration: run the whole plan under each candidate (tile, stages,
-    zunroll) with per-group CUDA-event timing and keep, for every group, its fastest legal
+    zunroll, ...) with per-group CUDA-event timing and keep, for every group, its fastest legal
     candidate.  Mutates the arrays (they are synthetic; the timed runs start from the result)."""
     import torch
     import paper_conf_sc_wahibm14_b200 as kf
     best = None
     tried = []
     for cand in AUTOTUNE_CANDIDATES:
-        tile, stages, zu, ru, mb, cl = cand[:6]
-        pb = cand[6] if len(cand) > 6 else 1
-        zq = cand[7] if len(cand) > 7 else 1
-        kw = dict(base_kw)
-        kw.update(tile=tile, stages=stages, zunroll=zu, ringunroll=ru, minblocks=mb, canvas_ld=cl, pblock=(pb, 1), pair_zq=zq)
-        tgt = kf.Target(**kw)
+        kw = cand_kw(base_kw, cand)
         try:
-            ex = kf.Exec(prog, plan, tgt)
+            ex = kf.Exec(prog, plan, kf.Target(**kw))
         except Exception:
             continue
         sb = ex.scratch_bytes()
@@ -308,13 +451,11 @@ def autotune(prog, plan, dev, base_kw, steps=6):
         gms, _ = ex.group_times()
         tried.append((tuple(cand), [g / steps for g in gms]))
         if best is None:
-            best = [(g / steps, kw) for g in gms]
+            best = [(g / steps, kw, cand) for g in gms]
         else:
-            best = [min(b, (g / steps, kw), key=lambda v: v[0]) for b, g in zip(best, gms)]
+            best = [min(b, (g / steps, kw, cand), key=lambda v: v[0]) for b, g in zip(best, gms)]
         del ex, scr
-    return ([kf.Target(**kw) for _, kw in best],
-            [(list(kw["tile"]), kw["stages"], kw["zunroll"], kw["ringunroll"], kw["minblocks"], kw["canvas_ld"],
-              kw["pblock"][0], kw["pair_zq"]) for _, kw in best], tried)
+    return [kf.Target(**kw) for _, kw, _ in best], [cand_norm(c) for _, _, c in best], tried
 
 
 def max_over_ranks(x: float) -> float:
@@ -374,8 +515,49 @@ def time_runner(rn, dev, steps, warmup, stream, profile=False, clk=None):
     return ms, gt
 
 
-def grid_for(world):
-    return {1: (1, 1), 2: (2, 1), 4: (2, 2), 8: (4, 2)}.get(world, (world, 1))
+def parity_windows(wl, prog, rn, rank, world, stream, nsteps=2, w=8):
+    """Parity of the configuration just timed: fresh seeded inputs, `nsteps` steps through the same
+    executor (plan and per-group launch configurations), then windows compared with the oracle on
+    dependency-cone crops (oracle/windows.py).  N = 1: windows anywhere (periodic seams, corners,
+    tile edges); N > 1: windows deep inside the rank's sub-domain (the cone stays local)."""
+    import numpy as np
+    import torch
+    import paper_conf_sc_wahibm14_b200 as kf
+    from oracle import graph, interp
+    from oracle.windows import crop, crop_window, dependency_radius, window
+    desc = wl.desc
+    if wl.gen not in ("weather", "uniform", "fig3"):
+        return {"skipped": f"inputs of workload {wl.name} are generated on the device"}
+    dev, host_in = wl.inputs(prog, rank)
+    rn.run(dev, nsteps, stream)
+    torch.cuda.synchronize()
+    got = kf.host_arrays(prog, dev)
+    del dev
+    M = dependency_radius(desc, nsteps) + 1
+    nx, ny, _ = desc.n
+    if world == 1:
+        pos = [(0, 0), (nx - 4, 3), (nx // 2 - 4, ny - 5), (131 % nx, 257 % ny), (nx - w, ny - w), (64 % nx, 64 % ny)]
+    else:
+        pos = [(M + 1, M + 1), (nx // 2, ny // 2), (nx - M - w - 1, ny - M - w - 1)]
+    names = [nm for x, (nm, _) in enumerate(desc.arrays)
+             if not graph.writers(desc, x) or graph.step_live(desc, x)]
+    t0 = time.perf_counter()
+    ok, bad = 0, []
+    for (x0, y0) in pos:
+        sub, sin = crop(desc, host_in, x0, y0, w, M)
+        ref = interp.run(sub, sin, nsteps)
+        for nm in names:
+            r = crop_window(sub, ref[nm], w, M)
+            g_ = window(desc, got[nm], x0, y0, w)
+            bt = np.uint32 if r.dtype == np.float32 else np.uint64
+            if np.array_equal(g_.view(bt), r.view(bt)):
+                ok += 1
+            else:
+                bad.append([nm, x0, y0])
+    return {"windows": len(pos), "window": f"{w}x{w}x{desc.n[2]}", "steps": nsteps, "arrays": names,
+            "compared": ok + len(bad), "bit_exact": not bad, "mismatches": bad[:8], "margin": M,
+            "oracle_s": round(time.perf_counter() - t0, 2),
+            "method": "oracle/windows.py dependency-cone crops of fresh seeded inputs, same executor as timed"}
 
 
 def run_kf(args):
@@ -387,23 +569,34 @@ def run_kf(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        raise SystemExit(f"bench.py: WORLD_SIZE={world} but --gpus {args.gpus}")
     if world > 1:
         torch.cuda.set_device(local)
         torch.distributed.init_process_group("nccl", device_id=torch.device("cuda", local))
     else:
         torch.cuda.set_device(0)
-    desc, gen, tkw, label = workload(args.workload)
+    wl = Workload(args.workload, world)
+    desc = wl.desc
     if args.relax_all and desc.name == "weather":
-        desc = desc.with_(flags=PROG_RELAX_ALL)
+        desc = wl.desc = desc.with_(flags=PROG_RELAX_ALL)
+    tkw = dict(wl.tkw)
     if args.tile:
         tkw["tile"] = tuple(int(v) for v in args.tile.split(","))
     if args.stages:
         tkw["stages"] = args.stages
     if args.threads:
         tkw["threads"] = args.threads
+    # single domain: the producing groups write the periodic ghost copies (no ghost-fill launches);
+    # decomposed: halo exchanges replace the fills
+    tkw["ghostwrite"] = 1 if (world == 1 and not args.fills) else 0
+    if world > 1:
+        px, py = grid_for(world)
+        tkw["internal_axes"] = (1 if px > 1 else 0) | (2 if py > 1 else 0)
     target = kf.Target(**tkw)
-    prog = kf.Program(desc)          # the per-GPU sub-domain program (weak scaling)
+    prog = kf.Program(desc)          # the per-GPU sub-domain program
     plan, plan_kind = (None, None) if args.plan == "select" else choose_plan(prog, target, args.plan)
+
     def new_dist_info():
         """A fresh NCCL unique id (broadcast from rank 0) for every communicator kf.Dist creates."""
         if world == 1:
@@ -413,17 +606,7 @@ def run_kf(args):
         t = torch.tensor(list(nid), dtype=torch.uint8, device="cuda")
         torch.distributed.broadcast(t, 0)
         return (px, py, rank, world, bytes(t.cpu().tolist()))
-    # synthetic inputs of the paper-shaped workload (seed 3 + rank: each rank owns its sub-domain)
-    if gen is None:
-        # large uniform workloads: U[-1,1) generated on the device (seeded torch generator)
-        L = prog.layout()
-        gdev = torch.Generator(device="cuda").manual_seed(3 + rank)
-        dt = torch.float64 if desc.dtype == 1 else torch.float32
-        dev = [torch.rand(L.elems, generator=gdev, device="cuda", dtype=dt) * 2 - 1 for _ in desc.arrays]
-    else:
-        inputs = gen(desc, 3 + rank)
-        dev = kf.device_arrays(prog, inputs)
-        del inputs
+    dev, _ = wl.inputs(prog, rank)
     stream = torch.cuda.current_stream()
     t0 = time.time()
     candidates, ranked = None, []
@@ -437,12 +620,7 @@ def run_kf(args):
     tuned, gtargets, tried = None, None, None
     if args.tuned:   # fixed per-group configs (e.g. for an ncu run of exactly the timed configuration)
         tuned = json.loads(args.tuned)
-        gtargets = [kf.Target(**dict(tkw, tile=tuple(c[0]), stages=c[1], zunroll=c[2], ringunroll=c[3],
-                                            minblocks=c[4] if len(c) > 4 else 0,
-                                            canvas_ld=c[5] if len(c) > 5 else 1,
-                                            pblock=(c[6] if len(c) > 6 else 1, 1),
-                                            pair_zq=c[7] if len(c) > 7 else 1))
-                    for c in tuned]
+        gtargets = [kf.Target(**cand_kw(tkw, c)) for c in tuned]
     elif args.autotune:
         if rank == 0:
             gtargets, tuned, tried = autotune(prog, plan, dev, tkw)
@@ -459,16 +637,10 @@ def run_kf(args):
             obj = [tuned]
             torch.distributed.broadcast_object_list(obj, 0)
             tuned = obj[0]
-            gtargets = [kf.Target(**dict(tkw, tile=tuple(c[0]), stages=c[1], zunroll=c[2], ringunroll=c[3],
-                                            minblocks=c[4] if len(c) > 4 else 0,
-                                            canvas_ld=c[5] if len(c) > 5 else 1,
-                                            pblock=(c[6] if len(c) > 6 else 1, 1),
-                                            pair_zq=c[7] if len(c) > 7 else 1))
-                        for c in tuned]
+            gtargets = [kf.Target(**cand_kw(tkw, c)) for c in tuned]
     rn = Runner(prog, plan, target, gtargets, new_dist_info())
     jit_s = time.time() - t0
     info = rn.ex.info()
-    npts = desc.npts
 
     with ClockSampler(local) as clk:
         ms, _ = time_runner(rn, dev, args.steps, args.warmup, stream, clk=clk)
@@ -476,17 +648,22 @@ def run_kf(args):
     clocks = clk.summary()
     # per-group device times over a second timed region (events on the launch stream)
     ms_prof, (gms, nlaunch) = time_runner(rn, dev, args.steps, 1, stream, profile=True)
-    # unfused plan on the same inputs: speedup vs unfused
+    # unfused plan on the same inputs: speedup vs unfused, and the original per-kernel times
     unf = None
+    k_ms = None
     if not args.no_unfused and args.plan != "unfused":
-        rn_u = Runner(prog, list(range(prog.nk)), target, None, new_dist_info())
+        ut = kf.Target(**dict(tkw))
+        rn_u = Runner(prog, list(range(prog.nk)), ut, None, new_dist_info())
         ms_u, _ = time_runner(rn_u, dev, args.steps, args.warmup, stream)
         ms_u = max_over_ranks(ms_u)
-        unf = {"ms_per_step": ms_u / args.steps, "bytes_per_step": rn_u.ex.info().compulsory_bytes_per_step}
+        _, (kms, _) = time_runner(rn_u, dev, args.steps, 1, stream, profile=True)
+        k_ms = [v / args.steps for v in kms]
+        unf = {"ms_per_step": ms_u / args.steps, "bytes_per_step": rn_u.ex.info().compulsory_bytes_per_step,
+               "launches_per_step": rn_u.ex.info().launches_per_step}
         del rn_u
     # end-to-end through the public API with host buffers (copies inside the timed region)
     e2e = None
-    if not args.no_e2e and gen is not None:
+    if not args.no_e2e and wl.gen not in ("device_uniform", "weather_tiled"):
         k = max(1, min(args.steps, 3))
         if rn.dist is None:
             host = [t.cpu().pin_memory() for t in dev]
@@ -517,15 +694,15 @@ def run_kf(args):
             d2h = sum(host[x].numel() * host[x].element_size() for x in outs)
             how = "kf.Dist.run with pinned host buffers copied in/out every step, host wall clock"
         dt = max_over_ranks(dt)
-        e2e = {"value": world * npts * k / dt, "unit": UNIT, "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+        e2e = {"value": wl.global_npts * k / dt, "unit": UNIT, "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
                "steps": k, "timing": how + ", max over ranks"}
         del host
 
     bytes_step = info.compulsory_bytes_per_step
-    value = world * npts * args.steps / (ms / 1e3)
+    value = wl.global_npts * args.steps / (ms / 1e3)
     peaks = measured_peaks()
     hbm_peak = peaks["hbm_gbs"] if peaks and "hbm_gbs" in peaks else 6650.0
-    peak_src = "MEASURED_PEAKS.json hbm_gbs" if peaks else "B200_PROFILING.md fallback 6.65 TB/s"
+    peak_src = "MEASURED_PEAKS.json hbm_gbs (burst copy)" if peaks else "B200_PROFILING.md fallback 6.65 TB/s"
     g_dom = int(np.argmax(gms))
     gi = rn.ex.group_info(g_dom)
     gname = gi.name.decode() if isinstance(gi.name, bytes) else gi.name
@@ -537,18 +714,50 @@ def run_kf(args):
                 "algorithmic_bytes_per_launch": gi.bytes_per_launch,
                 "per_group_ms_per_step": [g / args.steps for g in gms]}
     achieved_step = bytes_step / (ms / args.steps / 1e3) / 1e9
+    # NEXT-2 (Figs. 6-8 analogue): per group measured vs projected vs the original kernels' sum
+    per_groups = []
+    canon = []
+    m_ = {}
+    for g in plan:
+        canon.append(m_.setdefault(g, len(m_)))
+    tgt_of = gtargets if gtargets else [target] * len(gms)
+    for g in range(len(gms)):
+        per_g, _, _ = prog.project(plan, tgt_of[g])
+        gi_ = rn.ex.group_info(g)
+        ks = [k for k in range(prog.nk) if canon[k] == g]
+        row = {"group": g, "kernel": gi_.name.decode() if isinstance(gi_.name, bytes) else gi_.name,
+               "kernels": len(ks), "measured_ms": gms[g] / args.steps,
+               "t_model_ms": per_g[g].t_model_s * 1e3,
+               "t_bytes_ms": (per_g[g].bytes_read + per_g[g].bytes_written) / (hbm_peak * 1e9) * 1e3,
+               "original_sum_ms": sum(k_ms[k] for k in ks) if k_ms else None,
+               "regs": gi_.regs, "regs_est": per_g[g].regs_est, "smem": gi_.smem_bytes,
+               "threads": gi_.threads, "frac_of_copy_peak": gi_.bytes_per_launch / (gms[g] / args.steps / 1e3) / 1e9 / hbm_peak}
+        per_groups.append(row)
+    mod_err = [abs(r["t_model_ms"] / r["measured_ms"] - 1) for r in per_groups if r["measured_ms"] > 0]
     per, _, t_proj = prog.project(plan, target)
+    parity = None
+    if not args.no_parity:
+        parity = parity_windows(wl, prog, rn, rank, world, stream)
+        if world > 1:
+            obj = [parity]
+            allp = [None] * world
+            torch.distributed.all_gather_object(allp, parity)
+            parity = {"ranks": allp, "bit_exact": all(p_.get("bit_exact", False) for p_ in allp if "skipped" not in p_)}
+    px, py = grid_for(world)
     res = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
-        "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": wl.scaling, "vs_baseline": None,
         "dtype": "f64" if desc.dtype == 1 else "f32", "data": "synthetic (seeded, paper-shaped fields)",
-        "config": {"workload": label + (" with RELAX_ALL renaming" if desc.flags & 2 else ""),
+        "config": {"workload": wl.label + (" with RELAX_ALL renaming" if desc.flags & 2 else ""),
                    "plan": f"{plan_kind}: {info.n_groups} fused groups of {prog.nk} kernels",
                    "plan_labels": plan, "tile": list(target.tile), "stages": target.stages,
-                   "threads": target.threads, "l2": "inputs larger than L2 (each array > 126 MB), no flush",
-                   "parallelism": (f"xy domain decomposition {grid_for(world)[0]}x{grid_for(world)[1]}, NCCL halo "
-                                   f"exchange, weak (512x512x128 per GPU)") if world > 1 else "1 GPU",
-                   "graph": world == 1, "jit_s": round(jit_s, 2),
+                   "threads": target.threads, "ghostwrite": tkw["ghostwrite"],
+                   "l2": "inputs larger than L2 (each array > 126 MB), no flush" if desc.npts * desc.es > 126e6
+                   else "inputs smaller than L2 (no flush; small config)",
+                   "parallelism": (f"xy domain decomposition {px}x{py}, NCCL halo exchange (batched per phase, "
+                                   f"overlapped with interior tiles, CUDA graph), {wl.scaling}") if world > 1 else "1 GPU",
+                   "local_grid": list(desc.n), "global_points": wl.global_npts,
+                   "graph": True, "jit_s": round(jit_s, 2),
                    "per_group_launch_config": tuned if tuned else "uniform",
                    "plan_candidates": candidates,
                    "autotune_tried": [{"config": list(c), "group_ms": [round(x, 4) for x in g]} for c, g in tried]
@@ -557,9 +766,13 @@ def run_kf(args):
         "frac_of_measured_copy": achieved_step / hbm_peak,
         "frac_of_nominal_8TBs": achieved_step / 8000.0,
         "compulsory_bytes_per_step": bytes_step,
+        "fills_per_step": info.fills_per_step,
         "projected_ms_per_step": t_proj * 1e3,
         "model_ms_per_step": sum(g.t_model_s for g in per) * 1e3,
+        "per_group": per_groups,
+        "model_error_max": max(mod_err) if mod_err else None,
         "roofline": roofline,
+        "parity": parity,
         "gpu_launches": int(info.launches_per_step * args.steps),
         "clocks": clocks,
     }
@@ -580,43 +793,92 @@ def run_kf(args):
         torch.distributed.destroy_process_group()
 
 
+def run_all_plans(args):
+    """Config 2: every legal plan of the suite program at 256^3 timed on one GPU
+    (JIT of all plans on parallel host threads, identical groups compiled once), reporting the
+    best, the worst, the unfused plan and Fusion Efficiency; one JSON line with every plan."""
+    import torch
+    from concurrent.futures import ThreadPoolExecutor
+    import paper_conf_sc_wahibm14_b200 as kf
+    torch.cuda.set_device(0)
+    wl = Workload(args.workload, 1)
+    tkw = dict(wl.tkw, ghostwrite=1)
+    target = kf.Target(**tkw)
+    prog = kf.Program(wl.desc)
+    plans = prog.legal_plans(target)
+    dev, _ = wl.inputs(prog, 0)
+    t0 = time.time()
+    with ThreadPoolExecutor(max_workers=min(32, os.cpu_count() or 4)) as pool:
+        execs = list(pool.map(lambda pl: kf.Exec(prog, pl, target), plans))
+    jit_s = time.time() - t0
+    rows = []
+    for pl, ex in zip(plans, execs):
+        ms = time_exec(ex, dev, args.steps, warm=args.warmup)
+        b = ex.info().compulsory_bytes_per_step
+        rows.append({"plan": pl, "groups": len(set(pl)), "ms_per_step": ms, "bytes_per_step": b,
+                     "proj_ms": prog.project(pl, target)[2] * 1e3})
+    del execs
+    unf = [r for r in rows if r["groups"] == prog.nk][0]
+    best = min(rows, key=lambda r: r["ms_per_step"])
+    worst = max(rows, key=lambda r: r["ms_per_step"])
+    fe = lambda r: (r["bytes_per_step"] / unf["bytes_per_step"]) / (r["ms_per_step"] / unf["ms_per_step"])  # noqa: E731
+    npts = wl.desc.npts
+    out = {"metric": METRIC, "value": npts / (best["ms_per_step"] / 1e3), "unit": UNIT, "n_gpus": 1,
+           "steps": args.steps, "warmup": args.warmup, "ms_per_step": best["ms_per_step"], "higher_is_better": True,
+           "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+           "config": {"workload": wl.label, "mode": "every legal plan timed (P:435, P:481)", "legal_plans": len(rows),
+                      "tile": list(target.tile), "jit_s": round(jit_s, 1)},
+           "best": dict(best, fusion_efficiency=fe(best), speedup_vs_unfused=unf["ms_per_step"] / best["ms_per_step"]),
+           "worst": dict(worst, fusion_efficiency=fe(worst), speedup_vs_unfused=unf["ms_per_step"] / worst["ms_per_step"]),
+           "unfused": unf,
+           "projection_rank_corr": None,
+           "plans": rows}
+    try:
+        import numpy as np
+        a = np.argsort(np.argsort([r["proj_ms"] for r in rows]))
+        b = np.argsort(np.argsort([r["ms_per_step"] for r in rows]))
+        out["projection_rank_corr"] = float(np.corrcoef(a, b)[0, 1])
+    except Exception:
+        pass
+    print(json.dumps(out))
+
+
 def run_reference(args):
-    """--impl reference: the oracle as it stands on the host cores (rank 0 only)."""
+    """--impl reference: the oracle as it stands on the host cores (rank 0 only), a bounded
+    sub-grid sample of the same workload per timed step."""
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
     from oracle import interp
-    from workloads import programs, data
-    desc, gen, tkw, label = workload(args.workload)
-    # bounded sample of the same workload: a sub-grid, one oracle step per timed step
-    if args.workload.startswith("weather"):
-        sub = programs.weather(n=(64, 64, 128))
-        sample = "weather program on a 64x64x128 sub-grid of the 512x512x128 workload, 1 step per timed step"
-    elif args.workload == "tiny":
-        sub = desc
-        sample = "tiny 32^3 (full workload)"
-    elif args.workload == "fig3":
-        sub = programs.fig3(n=(64, 64, 128))
-        sample = "fig3 on a 64x64x128 sub-grid"
-    else:
-        sub = programs.stress(m=2, n=(64, 64, 64))
-        sample = "stress on a 64^3 sub-grid"
-    inp = gen(sub, 3)
+    desc, inp, sample = _oracle_sample(args.workload)
+    wl_label = Workload(args.workload, 1).label if args.workload != "stress" else "config 5 stress"
     for _ in range(args.warmup):
-        inp = interp.run(sub, inp, 1)
+        inp = interp.run(desc, inp, 1)
     t0 = time.perf_counter()
     for _ in range(args.steps):
-        inp = interp.run(sub, inp, 1)
+        inp = interp.run(desc, inp, 1)
     dt = time.perf_counter() - t0
-    value = sub.npts * args.steps / dt
+    value = desc.npts * args.steps / dt
     res = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": int(os.environ.get("WORLD_SIZE", "1")),
            "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3,
            "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
            "dtype": "f64" if desc.dtype == 1 else "f32", "data": "synthetic", "impl": "reference",
-           "config": {"workload": label},
-           "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+           "config": {"workload": wl_label},
+           "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
+                            "sample": sample + ", 1 step per timed step (numpy oracle, unfused)"},
            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(res))
+
+
+def relaunch_distributed(n: int) -> int:
+    """--gpus N > 1 without a launcher: one rank per GPU under torch.distributed.run."""
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
 
 
 def main():
@@ -633,18 +895,31 @@ def main():
     ap.add_argument("--tile", default=None)
     ap.add_argument("--stages", type=int, default=None)
     ap.add_argument("--threads", type=int, default=None)
+    ap.add_argument("--fills", action="store_true", help="ghost-fill launches instead of ghost writes (A/B)")
+    ap.add_argument("--all-plans", action="store_true", help="time every legal plan (programs of <= 14 kernels)")
     ap.add_argument("--no-unfused", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-parity", action="store_true")
     ap.add_argument("--autotune", type=int, default=1, help="per-group launch configuration by measurement (1/0)")
-    ap.add_argument("--tuned", default=None, help="JSON per-group configs [[tile,stages,zunroll,ringunroll(,minblocks)],...] "
-                                                  "(skips autotune; as printed in config.per_group_launch_config: "
-                                                  "[tile, stages, zunroll, ringunroll, minblocks, canvas_ld, pblock_x, pair_zq])")
+    ap.add_argument("--tuned", default=None, help="JSON per-group configs as printed in config.per_group_launch_config: "
+                                                  "[tile, stages, zunroll, ringunroll, minblocks, canvas_ld, pblock_x, pair_zq]")
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "kf":
         args.warmup = 3
     if args.impl == "reference":
         run_reference(args)
+        return
+    if args.gpus < 1:
+        raise SystemExit("--gpus must be >= 1")
+    if "WORLD_SIZE" not in os.environ and args.gpus > 1:
+        import torch
+        have = torch.cuda.device_count()
+        if have < args.gpus:
+            raise SystemExit(f"bench.py: --gpus {args.gpus} but only {have} CUDA device(s) visible")
+        sys.exit(relaunch_distributed(args.gpus))
+    if args.all_plans:
+        run_all_plans(args)
     else:
         run_kf(args)
 

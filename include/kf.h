@@ -138,6 +138,9 @@ kf_status kf_program_reach(const kf_program* prog, uint8_t* reach);
 typedef enum { KF_CLS_RO = 0, KF_CLS_RW = 1, KF_CLS_EXPANDABLE = 2, KF_CLS_WO = 3 } kf_array_class;
 typedef struct { int32_t cls, n_writers, n_readers, relaxed, step_live, upward_exposed; } kf_array_info;
 kf_status kf_program_array_info(const kf_program* prog, int32_t array, kf_array_info* out);
+/* The class of every array at once: cls[n_arrays] (caller-owned) receives kf_array_class values
+ * (SURVEY 8(b)). */
+kf_status kf_program_array_class(const kf_program* prog, int32_t* cls);
 
 /* Degree of kinship (Table II) of kernels a and b inside `group` (R5: the chain
  * must stay inside the group; 0 if none). */
@@ -271,6 +274,11 @@ kf_status kf_plan_search(const kf_program* prog, const kf_target* target, int32_
                          uint64_t seed, int32_t* plan_out, uint64_t* bytes_out);
 /* Number of legal partitions (brute force; n <= 14). */
 kf_status kf_plan_count_legal(const kf_program* prog, const kf_target* target, uint64_t* count);
+/* Every legal partition (brute force over restricted-growth strings, n <= 14) in enumeration order:
+ * plans[i*n .. i*n+n) = canonical labels of the i-th legal plan for i < cap; *count = the total
+ * (call with cap = 0 to size the buffer).  Config 2 "every legal plan run". */
+kf_status kf_plan_enumerate(const kf_program* prog, const kf_target* target, int32_t* plans, int64_t cap,
+                            int64_t* count);
 
 /* ------------------------------------------------------------------ execution (sm_100a) */
 typedef struct kf_exec kf_exec;
@@ -330,6 +338,11 @@ kf_status kf_exec_set_profiling(kf_exec* ex, int32_t on);
 kf_status kf_exec_group_times(kf_exec* ex, double* ms, int32_t cap, int32_t* n, int64_t* launches);
 /* Use a captured CUDA graph for the step loop (default on). */
 kf_status kf_exec_set_graph(kf_exec* ex, int32_t on);
+/* The caller changed array contents outside the interior (e.g. FROZEN ghost values) while keeping
+ * the same device pointers: the next run re-copies them into the renamed scratch versions (R9).
+ * Without this call, FROZEN ghost values must stay constant for a given pointer set.
+ * (kf_run_host does it itself after every upload.) */
+kf_status kf_exec_invalidate(kf_exec* ex);
 
 /* ------------------------------------------------------------------ multi-GPU (row a11) */
 /* Domain decomposition over a px x py process grid (x, y split; z whole; part/rank index
@@ -357,7 +370,38 @@ kf_status kf_dist_run(kf_dist* d, void* const* arrays, void* const* scratch, uin
  * cuda_stream; the other tiles are launched after the exchanges complete.  Results are
  * identical either way; off = exchanges and whole-group launches in stream order. */
 kf_status kf_dist_set_overlap(kf_dist* d, int32_t on);
+/* Capture one replay period of kf_dist_run (exchanges, overlap and NCCL calls included) in a CUDA
+ * graph (default on; if the capture fails the dist runs eagerly from then on). */
+kf_status kf_dist_set_graph(kf_dist* d, int32_t on);
+/* Halo strip geometry of the LOCAL program on a decomposed axis (0 = x, 1 = y), in elements of
+ * kf_array_layout: out[0] send_lo (first ghost-deep interior strip, goes to the low neighbour's
+ * high ghost), out[1] send_hi, out[2] recv_lo (low ghost), out[3] recv_hi.  x strips cover every
+ * padded row; y strips are whole padded rows (x ghosts = corners included). */
+typedef struct { int64_t offset; int32_t w, h, d, pad; } kf_box;
+kf_status kf_dist_strips(const kf_program* prog, int32_t axis, kf_box out[4]);
 void kf_dist_destroy(kf_dist* d);
+
+/* ------------------------------------------------------------------ §8(b) one-call interface
+ * The problem statement's boundary (Fig. 4): a program, a plan F (group label per kernel),
+ * the data arrays D -- run N timesteps.  kf_run keeps one kf_exec per (device, canonical plan)
+ * inside the program handle (validated, lowered and JIT-compiled on the first call for that plan
+ * with the kf_target_b200 defaults; freed by kf_program_destroy), so repeated calls only launch.
+ *
+ * kf_scratch_bytes: device scratch kf_run needs for `plan` (one buffer per renamed version,
+ * P:53; it depends on the program only, plan may be NULL).
+ * kf_run: arrays = n_arrays caller-owned device pointers (allocation bases, kf_array_layout,
+ * 128-byte aligned); scratch >= kf_scratch_bytes; params = n_params values (NULL if none);
+ * asynchronous on cuda_stream.  Results/errors as kf_exec_run (KF_E_ILLEGAL_PLAN for an illegal
+ * plan, KF_E_NVRTC if the JIT fails).  Not thread-safe per program.
+ * kf_dist_init: makes later kf_run calls on this program distributed over a px x py process grid
+ * (rank = iy*px + ix, world = px*py, the program describing the LOCAL sub-domain with PERIODIC
+ * decomposed axes): halo exchange by NCCL over NVLink replaces the periodic wrap (row a11).  id =
+ * kf_dist_unique_id() of rank 0, broadcast by the caller; ignored when world == 1.  Once per
+ * program; KF_E_NCCL if the communicator cannot be created. */
+kf_status kf_scratch_bytes(const kf_program* prog, const int32_t* plan, uint64_t* bytes);
+kf_status kf_run(kf_program* prog, const int32_t* plan, void* const* arrays, void* scratch, uint64_t scratch_bytes,
+                 int64_t nsteps, const double* params, void* cuda_stream);
+kf_status kf_dist_init(kf_program* prog, int32_t rank, int32_t world, int32_t px, int32_t py, const uint8_t id[128]);
 
 /* ------------------------------------------------------------------ utilities */
 /* Overwrite `bytes` of caller-provided device memory on `cuda_stream` (benchmarks: evict

@@ -95,6 +95,10 @@ class kf_group_info(C.Structure):
                 ("bytes_per_launch", C.c_uint64), ("name", C.c_char * 64)]
 
 
+class kf_box(C.Structure):
+    _fields_ = [("offset", C.c_int64), ("w", C.c_int32), ("h", C.c_int32), ("d", C.c_int32), ("pad", C.c_int32)]
+
+
 class kf_paper_meta(C.Structure):
     _fields_ = [(n, C.c_int32) for n in ("t_b", "blocks_smx", "thr", "blocks", "hal", "halo", "shared_arrays", "smx",
                                          "r_t", "r_max", "r_smx", "r_adr", "sh_smx", "b_conf", "elem_bytes", "pad")] + \
@@ -120,6 +124,7 @@ SIGNATURES = {
     "kf_program_edges": (C.c_int, [P, C.POINTER(kf_edge), C.c_int32, I32P]),
     "kf_program_reach": (C.c_int, [P, C.POINTER(C.c_uint8)]),
     "kf_program_array_info": (C.c_int, [P, C.c_int32, C.POINTER(kf_array_info)]),
+    "kf_program_array_class": (C.c_int, [P, I32P]),
     "kf_program_kinship": (C.c_int, [P, C.c_int32, C.c_int32, I32P, C.c_int32, I32P]),
     "kf_array_layout": (C.c_int, [P, C.POINTER(kf_layout)]),
     "kf_target_b200": (C.c_int, [C.POINTER(kf_target)]),
@@ -131,6 +136,7 @@ SIGNATURES = {
                                     C.c_int32, I32P]),
     "kf_plan_search": (C.c_int, [P, C.POINTER(kf_target), C.c_int32, C.c_uint64, I32P, U64P]),
     "kf_plan_count_legal": (C.c_int, [P, C.POINTER(kf_target), U64P]),
+    "kf_plan_enumerate": (C.c_int, [P, C.POINTER(kf_target), I32P, C.c_int64, C.POINTER(C.c_int64)]),
     "kf_exec_create": (C.c_int, [P, I32P, C.POINTER(kf_target), C.POINTER(P)]),
     "kf_exec_create_ex": (C.c_int, [P, I32P, C.POINTER(kf_target), C.c_int32, C.POINTER(P)]),
     "kf_exec_destroy": (None, [P]),
@@ -143,6 +149,7 @@ SIGNATURES = {
     "kf_exec_set_profiling": (C.c_int, [P, C.c_int32]),
     "kf_exec_group_times": (C.c_int, [P, C.POINTER(C.c_double), C.c_int32, I32P, C.POINTER(C.c_int64)]),
     "kf_exec_set_graph": (C.c_int, [P, C.c_int32]),
+    "kf_exec_invalidate": (C.c_int, [P]),
     "kf_flush_l2": (C.c_int, [P, C.c_uint64, P]),
     "kf_paper_projection": (C.c_int, [C.POINTER(kf_paper_meta), C.POINTER(kf_paper_proj)]),
     "kf_dist_unique_id": (C.c_int, [C.POINTER(C.c_uint8)]),
@@ -152,6 +159,11 @@ SIGNATURES = {
     "kf_dist_run": (C.c_int, [P, C.POINTER(P), C.POINTER(P), C.c_uint64, C.c_int64, C.POINTER(C.c_double), P]),
     "kf_dist_set_overlap": (C.c_int, [P, C.c_int32]),
     "kf_dist_destroy": (None, [P]),
+    "kf_dist_set_graph": (C.c_int, [P, C.c_int32]),
+    "kf_dist_strips": (C.c_int, [P, C.c_int32, C.POINTER(kf_box)]),
+    "kf_dist_init": (C.c_int, [P, C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.POINTER(C.c_uint8)]),
+    "kf_scratch_bytes": (C.c_int, [P, I32P, U64P]),
+    "kf_run": (C.c_int, [P, I32P, C.POINTER(P), P, C.c_uint64, C.c_int64, C.POINTER(C.c_double), P]),
     "kf_jit_check": (C.c_int, [P, I32P, C.POINTER(kf_target), C.c_int32, I32P, I32P, C.c_char_p, C.c_int64]),
 }
 

@@ -8,7 +8,7 @@ from typing import Dict, List, Optional, Sequence, Tuple
 
 import numpy as np
 
-from ._abi import (check, kf_access, kf_array_desc, kf_array_info, kf_edge, kf_exec_info, kf_group_info,
+from ._abi import (check, kf_access, kf_array_desc, kf_array_info, kf_box, kf_edge, kf_exec_info, kf_group_info,
                    kf_group_proj, kf_insn, kf_kernel_desc, kf_kernel_sched, kf_layout, kf_program_desc,
                    kf_program_info, kf_stmt, kf_target, kf_violation, lib)
 
@@ -128,6 +128,11 @@ class Program:
         check(lib().kf_program_array_info(self.h, x, C.byref(r)))
         return r
 
+    def array_classes(self) -> List[int]:
+        out = (C.c_int32 * self.na)()
+        check(lib().kf_program_array_class(self.h, out))
+        return list(out)
+
     def kinship(self, a: int, b: int, group: Sequence[int]) -> int:
         d = C.c_int32()
         check(lib().kf_program_kinship(self.h, a, b, _i32(group), len(group), C.byref(d)))
@@ -175,12 +180,50 @@ class Program:
         check(lib().kf_plan_count_legal(self.h, C.byref(t), C.byref(c)))
         return c.value
 
+    def legal_plans(self, target: Optional[Target] = None) -> List[List[int]]:
+        """Every legal partition (kf_plan_enumerate; n <= 14)."""
+        t = (target or Target()).c
+        n = C.c_int64()
+        check(lib().kf_plan_enumerate(self.h, C.byref(t), None, 0, C.byref(n)))
+        buf = (C.c_int32 * max(1, n.value * self.nk))()
+        check(lib().kf_plan_enumerate(self.h, C.byref(t), buf, n.value, C.byref(n)))
+        return [list(buf[i * self.nk:(i + 1) * self.nk]) for i in range(n.value)]
+
     def jit_check(self, plan, group, target: Optional[Target] = None):
         t = (target or Target()).c
         regs, spill = C.c_int32(), C.c_int32()
         log = C.create_string_buffer(1 << 16)
         check(lib().kf_jit_check(self.h, _i32(plan), C.byref(t), group, C.byref(regs), C.byref(spill), log, 1 << 16))
         return regs.value, spill.value, log.value.decode(errors="replace")
+
+    # ---- §8(b) one-call interface (kf_run / kf_scratch_bytes / kf_dist_init)
+    def scratch_bytes(self, plan: Optional[Sequence[int]] = None) -> int:
+        b = C.c_uint64()
+        check(lib().kf_scratch_bytes(self.h, _i32(plan) if plan is not None else None, C.byref(b)))
+        return b.value
+
+    def run(self, plan: Sequence[int], tensors, scratch, nsteps: int, params=None, stream=None):
+        """kf_run: JIT once per plan (cached in the program handle), then launch nsteps steps."""
+        import torch
+        if stream is None:
+            stream = torch.cuda.current_stream()
+        arr = (C.c_void_p * len(tensors))(*[t.data_ptr() for t in tensors])
+        sp = scratch.data_ptr() if scratch is not None else 0
+        sb = scratch.numel() * scratch.element_size() if scratch is not None else 0
+        prm = params if params is not None else self.desc.params
+        pr = (C.c_double * max(1, len(prm)))(*prm)
+        check(lib().kf_run(self.h, _i32(plan), arr, C.c_void_p(sp), sb, nsteps, pr, C.c_void_p(stream.cuda_stream)))
+
+    def dist_init(self, rank: int, world: int, px: int, py: int, nccl_id: Optional[bytes] = None):
+        idb = (C.c_uint8 * 128)(*nccl_id) if nccl_id is not None else None
+        check(lib().kf_dist_init(self.h, rank, world, px, py, idb))
+
+    def dist_strips(self, axis: int):
+        """Halo strips of this (local) program: [send_lo, send_hi, recv_lo, recv_hi] as
+        (offset, w, h, d) in elements of the kf layout (kf_dist_strips)."""
+        out = (kf_box * 4)()
+        check(lib().kf_dist_strips(self.h, axis, out))
+        return [(b.offset, b.w, b.h, b.d) for b in out]
 
     # ---- layout helpers (plumbing between the logical ghosted numpy layout and device memory)
     def to_device_layout(self, arr: np.ndarray) -> np.ndarray:
@@ -251,6 +294,10 @@ class Exec:
 
     def set_graph(self, on: bool):
         check(lib().kf_exec_set_graph(self.h, int(on)))
+
+    def invalidate(self):
+        """kf_exec_invalidate: array contents outside the interior changed under the same pointers."""
+        check(lib().kf_exec_invalidate(self.h))
 
     def group_times(self):
         n = C.c_int32()
@@ -329,13 +376,17 @@ class Dist:
         """Exchange / interior-compute overlap (kf_dist_set_overlap; default on)."""
         check(lib().kf_dist_set_overlap(self.h, 1 if on else 0))
 
+    def set_graph(self, on: bool):
+        """CUDA graph of one replay period (kf_dist_set_graph; default on)."""
+        check(lib().kf_dist_set_graph(self.h, 1 if on else 0))
+
     def run(self, part_tensors, part_scratch, nsteps: int, params=None, stream=None):
         import torch
         stream = stream or torch.cuda.current_stream()
         ptrs = [t.data_ptr() for ts in part_tensors for t in ts]
         arr = (C.c_void_p * len(ptrs))(*ptrs)
         scr = [s.data_ptr() if s is not None else 0 for s in part_scratch]
-        sb = min([s.numel() for s in part_scratch if s is not None] or [0])
+        sb = min([s.numel() * s.element_size() for s in part_scratch if s is not None] or [0])
         sarr = (C.c_void_p * len(scr))(*scr)
         prm = params if params is not None else self.parts[0].program.desc.params
         pr = (C.c_double * max(1, len(prm)))(*prm)

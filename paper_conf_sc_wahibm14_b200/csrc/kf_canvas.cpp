@@ -59,7 +59,7 @@ CanvasPlan plan_canvas(const Program& p, const GroupLowering& L) {
   // pair mode: pairs aligned to even tile-relative x (TX and NX even), so a pair never straddles
   // the tile or domain edge; one pair per thread
   if (!alive.empty() && L.pblock[0] == 2 && L.pblock[1] == 1 && U == 1 && TX % 2 == 0 && p.n[0] % 2 == 0 &&
-      !L.ghost_write && !getenv("KF_NO_CANVAS")) {
+      !getenv("KF_NO_CANVAS")) {
     c.lop = (c.clo[0] + 1) / 2;
     c.hip = (c.chi[0] + 1) / 2;
     c.cwp = TX / 2 + c.lop + c.hip;

@@ -491,11 +491,13 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
                         // CS2R; g0 -14 %) but loads on lanes outside the regions: more wavefronts and
                         // bank conflicts on the halo warp (+25 % shared wavefronts), so it is a per-group
                         // launch knob chosen by measurement.
+                        // Every address must lie inside the slot being read (not merely inside the
+                        // rings): a slot is never written in the phase that reads it, while a
+                        // neighbouring ring or slot may be (compute-sanitizer racecheck, round 2).
                         const Ring& RR = L.rings[key.ring];
-                        const long long amin = RR.smem_off + (long long)key.off * p.es;
-                        const long long amax = RR.smem_off + (long long)(RR.slots - 1) * RR.plane_bytes +
-                                               ((long long)(CH - 1) * RR.px + (cv.cw - 1) + key.off + 1) * p.es;
-                        const bool nopred = L.canvas_ld && amin >= 0 && amax <= L.mbar_off;
+                        const long long amin = (long long)key.off * p.es;
+                        const long long amax = ((long long)(CH - 1) * RR.px + (cv.cw - 1) + key.off + 1) * p.es;
+                        const bool nopred = L.canvas_ld && amin >= 0 && amax <= RR.plane_bytes;
                         std::string ld = nopred ? acc
                                                 : "(ca" + rs + " && cx" + rs + " >= " + std::to_string(rc[0]) + " && cx" + rs + " < " +
                                                       std::to_string(rc[1]) + " && cy" + rs + " >= " + std::to_string(rc[2]) + " && cy" +
@@ -619,10 +621,10 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
     const auto& [ring, po, rel] = pk;
     const Ring& RR = L.rings[ring];
     const long long cxmin = -PSH, cxmax = 2LL * (cv.cwp - 1) - PSH;
-    const long long amin = RR.smem_off + (cxmin + rel) * p.es;
-    const long long amax = RR.smem_off + (long long)(RR.slots - 1) * RR.plane_bytes +
-                           ((long long)(CH - 1) * RR.px + cxmax + rel + 2) * p.es;
-    return L.canvas_ld && amin >= 0 && amax <= L.mbar_off;
+    // inside the slot being read (see the single-point canvas above)
+    const long long amin = (cxmin + rel) * p.es;
+    const long long amax = ((long long)(CH - 1) * RR.px + cxmax + rel + 2) * p.es;
+    return L.canvas_ld && amin >= 0 && amax <= RR.plane_bytes;
   };
   // z register queues of the pair canvas: a pair value (ring, po, rel) read at iteration t is the
   // value (ring, po + 1, rel) had at iteration t - 1 -- loaded then by the same thread, or computed
@@ -852,6 +854,38 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
         for (size_t si = 0; si < K.stmts.size(); si++) {
           const int oi = out_index(Ver{K.stmts[si].out, p.vw(k, K.stmts[si].out)});
           if (oi >= 0) o << "        *(real2*)&a.out[" << oi << "][gi] = real2{" << v0[si] << ", " << v1[si] << "};\n";
+        }
+        if (L.ghost_write) {
+          // periodic x/y ghost copies of the pair (edge tiles only): a y ghost row takes the pair as a
+          // vector (same x); x ghosts and corners point by point (the ghost width may be odd)
+          const bool px_ = p.bc[0] == KF_BC_PERIODIC, py_ = p.bc[1] == KF_BC_PERIODIC;
+          o << "        if (edge_tile) {\n";
+          o << "          const long long pb = (long long)" << pz << " * PLANE;\n";
+          o << "          const bool wy = " << (py_ ? "(cgy_r0 < GY || cgy_r0 >= NY - GY)" : "false") << ";\n";
+          o << "          const int gy2 = cgy_r0 < GY ? cgy_r0 + NY : cgy_r0 - NY;\n";
+          o << "          if (wy) {\n";
+          for (size_t si = 0; si < K.stmts.size(); si++) {
+            const int oi = out_index(Ver{K.stmts[si].out, p.vw(k, K.stmts[si].out)});
+            if (oi >= 0)
+              o << "            *(real2*)&a.out[" << oi << "][pb + (long long)gy2 * PITCH + cgx_r0] = real2{" << v0[si] << ", "
+                << v1[si] << "};\n";
+          }
+          o << "          }\n";
+          if (px_)
+            for (int j = 0; j < 2; j++) {
+              o << "          { const int gxj = cgx_r0 + " << j << ";\n";
+              o << "            if (gxj < GX || gxj >= NX - GX) {\n";
+              o << "              const int gx2 = gxj < GX ? gxj + NX : gxj - NX;\n";
+              for (size_t si = 0; si < K.stmts.size(); si++) {
+                const int oi = out_index(Ver{K.stmts[si].out, p.vw(k, K.stmts[si].out)});
+                if (oi < 0) continue;
+                const std::string& v = j ? v1[si] : v0[si];
+                o << "              a.out[" << oi << "][pb + (long long)cgy_r0 * PITCH + gx2] = " << v << ";\n";
+                o << "              if (wy) a.out[" << oi << "][pb + (long long)gy2 * PITCH + gx2] = " << v << ";\n";
+              }
+              o << "            }\n          }\n";
+            }
+          o << "        }\n";
         }
         o << "      }\n";
       }

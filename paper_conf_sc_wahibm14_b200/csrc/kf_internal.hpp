@@ -200,6 +200,13 @@ Split split_units(const Program& p, const GroupLowering& L);
 
 struct kf_program {
   kf::Program p;
+  // kf_run state (kf_runtime.cpp): per-plan executors and the kf_dist_init context, freed with
+  // the program
+  void* run_cache = nullptr;
+  void (*run_cache_free)(void*) = nullptr;
+  ~kf_program() {
+    if (run_cache && run_cache_free) run_cache_free(run_cache);
+  }
 };
 
 #define KF_TRY(...)                                       \

@@ -67,10 +67,12 @@ __global__ void fill_z(T* __restrict__ base, Geom g) {
 // is periodic) and the y-ghost rows over the x range not already covered (if y is periodic).
 struct FillList { void* base[kMaxFillBufs]; };
 
+// zghost: only the z ghost planes (2*gz of them) -- the run-start fill of renamed scratch versions,
+// whose interior planes are not written yet (their x/y ghosts are filled after their producer).
 template <typename T>
-__global__ void fill_xy_multi(FillList L, Geom g, int px, int py) {
+__global__ void fill_xy_multi(FillList L, Geom g, int px, int py, int zghost) {
   T* base = (T*)L.base[blockIdx.y];
-  const int NZ = g.nz + 2 * g.gz, NYp = g.ny + 2 * g.gy;
+  const int NZ = zghost ? 2 * g.gz : g.nz + 2 * g.gz, NYp = g.ny + 2 * g.gy;
   const long long nxs = px ? 2LL * g.gx * NYp * NZ : 0;                  // x-ghost columns
   const int x_lo = px ? 0 : -g.gx, x_w = px ? g.nx : g.nx + 2 * g.gx;    // y rows: x range not in nxs
   const long long nys = py ? (long long)x_w * 2 * g.gy * NZ : 0;
@@ -93,6 +95,7 @@ __global__ void fill_xy_multi(FillList L, Geom g, int px, int py) {
     }
     const int si = (px && (i < 0 || i >= g.nx)) ? (i < 0 ? i + g.nx : i - g.nx) : i;
     const int sj = (py && (j < 0 || j >= g.ny)) ? (j < 0 ? j + g.ny : j - g.ny) : j;
+    if (zghost && k >= 0) k += g.nz;   // planes -gz..-1, then nz..nz+gz-1
     const long long o = (long long)(k + g.gz) * g.plane + g.xoff;
     base[o + (long long)(j + g.gy) * g.pitch + i] = base[o + (long long)(sj + g.gy) * g.pitch + si];
   }
@@ -128,6 +131,22 @@ __global__ void copy_box(T* __restrict__ dst, long long dpitch, long long dplane
   }
 }
 
+// Many w x h x d box copies in one launch (blockIdx.y = box): the strips of every buffer of an
+// exchange phase are packed / unpacked / copied together (a11).  Box element counts fit 32 bits
+// (ghost-deep strips), so the index arithmetic is 32-bit (division by the box's w and h only).
+template <typename T>
+__global__ void copy_boxes(BoxList L) {
+  const BoxCopy& b = L.box[blockIdx.y];
+  T* __restrict__ dst = (T*)b.dst;
+  const T* __restrict__ src = (const T*)b.src;
+  const unsigned w = unsigned(b.w), wh = unsigned(b.w) * unsigned(b.h);
+  const unsigned total = wh * unsigned(b.d);
+  for (unsigned i = blockIdx.x * blockDim.x + threadIdx.x; i < total; i += gridDim.x * blockDim.x) {
+    const unsigned z = i / wh, r = i - z * wh, y = r / w, x = r - y * w;
+    dst[z * b.dplane + (long long)y * b.dpitch + x] = src[z * b.splane + (long long)y * b.spitch + x];
+  }
+}
+
 __global__ void flush_kernel(uint4* __restrict__ buf, long long n, unsigned v) {
   for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x)
     buf[i] = make_uint4(v, v + 1, v + 2, v + 3);
@@ -156,10 +175,12 @@ cudaError_t launch_fill(int axis, void* base, int es, const Geom& g, cudaStream_
   return cudaGetLastError();
 }
 
-cudaError_t launch_fill_xy_multi(void* const* bufs, int n, int px, int py, int es, const Geom& g, cudaStream_t s) {
+cudaError_t launch_fill_xy_multi(void* const* bufs, int n, int px, int py, int es, const Geom& g, cudaStream_t s,
+                                 int zghost) {
   if (!px && !py) return cudaSuccess;
-  const long long per = (px ? 2LL * g.gx * (g.ny + 2 * g.gy) : 0) * (g.nz + 2 * g.gz) +
-                        (py ? (long long)(px ? g.nx : g.nx + 2 * g.gx) * 2 * g.gy * (g.nz + 2 * g.gz) : 0);
+  const long long NZ = zghost ? 2 * g.gz : g.nz + 2 * g.gz;
+  const long long per = (px ? 2LL * g.gx * (g.ny + 2 * g.gy) : 0) * NZ +
+                        (py ? (long long)(px ? g.nx : g.nx + 2 * g.gx) * 2 * g.gy * NZ : 0);
   if (per == 0) return cudaSuccess;
   for (int b0 = 0; b0 < n; b0 += kMaxFillBufs) {
     const int m = n - b0 < kMaxFillBufs ? n - b0 : kMaxFillBufs;
@@ -168,8 +189,8 @@ cudaError_t launch_fill_xy_multi(void* const* bufs, int n, int px, int py, int e
     long long nb = (per + 255) / 256;
     const long long cap = (148LL * 16 + m - 1) / m;   // ~16 CTAs per SM over all buffers
     dim3 grid(unsigned(nb < cap ? nb : cap), unsigned(m));
-    if (es == 4) fill_xy_multi<float><<<grid, 256, 0, s>>>(L, g, px, py);
-    else fill_xy_multi<double><<<grid, 256, 0, s>>>(L, g, px, py);
+    if (es == 4) fill_xy_multi<float><<<grid, 256, 0, s>>>(L, g, px, py, zghost);
+    else fill_xy_multi<double><<<grid, 256, 0, s>>>(L, g, px, py, zghost);
   }
   return cudaGetLastError();
 }
@@ -189,6 +210,27 @@ cudaError_t launch_copy_box(void* dst, long long dpitch, long long dplane, const
   int nb = blocks_for(n);
   if (es == 4) copy_box<float><<<nb, 256, 0, s>>>((float*)dst, dpitch, dplane, (const float*)src, spitch, splane, w, h, d);
   else copy_box<double><<<nb, 256, 0, s>>>((double*)dst, dpitch, dplane, (const double*)src, spitch, splane, w, h, d);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_copy_boxes(const BoxCopy* boxes, int n, int es, cudaStream_t s) {
+  for (int b0 = 0; b0 < n; b0 += kMaxBoxes) {
+    const int m = n - b0 < kMaxBoxes ? n - b0 : kMaxBoxes;
+    BoxList L{};
+    long long most = 0;
+    for (int i = 0; i < m; i++) {
+      L.box[i] = boxes[b0 + i];
+      const long long e = (long long)L.box[i].w * L.box[i].h * L.box[i].d;
+      if (e >= (1LL << 32)) return cudaErrorInvalidValue;
+      most = e > most ? e : most;
+    }
+    if (most == 0) continue;
+    const long long nb = (most + 255) / 256;
+    const long long cap = (148LL * 8 + m - 1) / m;   // ~8 CTAs per SM over all boxes
+    dim3 grid(unsigned(nb < cap ? nb : cap), unsigned(m));
+    if (es == 4) copy_boxes<float><<<grid, 256, 0, s>>>(L);
+    else copy_boxes<double><<<grid, 256, 0, s>>>(L);
+  }
   return cudaGetLastError();
 }
 

@@ -281,6 +281,14 @@ kf_status kf_program_reach(const kf_program* prog, uint8_t* reach) {
   });
 }
 
+kf_status kf_program_array_class(const kf_program* prog, int32_t* cls) {
+  KF_TRY({
+    if (!prog || !cls) fail(KF_E_ARG, "null argument");
+    const Program& p = prog->p;
+    for (int x = 0; x < p.na; x++) cls[x] = p.cls[x];
+  });
+}
+
 kf_status kf_program_array_info(const kf_program* prog, int32_t x, kf_array_info* out) {
   KF_TRY({
     if (!prog || !out) fail(KF_E_ARG, "null argument");

@@ -12,9 +12,11 @@
 #include <nvrtc.h>
 
 #include <algorithm>
+#include <atomic>
 #include <cstring>
 #include <functional>
 #include <sstream>
+#include <thread>
 
 #include "kf_internal.hpp"
 #include "kf_kernels.hpp"
@@ -24,6 +26,7 @@ namespace kf {
 // ---------------------------------------------------------------- driver entry points
 struct Drv {
   CUresult (*moduleLoadData)(CUmodule*, const void*) = nullptr;
+  CUresult (*moduleUnload)(CUmodule) = nullptr;
   CUresult (*moduleGetFunction)(CUfunction*, CUmodule, const char*) = nullptr;
   CUresult (*funcSetAttribute)(CUfunction, CUfunction_attribute, int) = nullptr;
   CUresult (*funcGetAttribute)(int*, CUfunction_attribute, CUfunction) = nullptr;
@@ -52,6 +55,7 @@ static Drv& drv() {
       if (e != cudaSuccess || q != cudaDriverEntryPointSuccess) *fp = nullptr;
     };
     get("cuModuleLoadData", (void**)&d.moduleLoadData);
+    get("cuModuleUnload", (void**)&d.moduleUnload);
     get("cuModuleGetFunction", (void**)&d.moduleGetFunction);
     get("cuFuncSetAttribute", (void**)&d.funcSetAttribute);
     get("cuFuncGetAttribute", (void**)&d.funcGetAttribute);
@@ -144,6 +148,11 @@ static std::shared_ptr<Compiled> compile_cached(const std::string& src, const st
 // its own on-disk cache (seen on reused GPU boxes): the spill test above then never fires.  The
 // loader checks the function's local memory instead and comes here for the uncapped build.
 static std::shared_ptr<Compiled> compile_nocap(const std::string& src, const std::string& name) {
+  {
+    std::lock_guard<std::mutex> lk(g_cache_mu);
+    auto it = g_cubin_cache.find(src);
+    if (it != g_cubin_cache.end() && it->second->nocap) return it->second;
+  }
   auto c = std::make_shared<Compiled>(nvrtc_compile("#define KF_NO_MAXNREG 1\n" + src, name));
   c->nocap = true;
   std::lock_guard<std::mutex> lk(g_cache_mu);
@@ -195,6 +204,7 @@ struct kf_exec {
   std::vector<double> cur_params;
   std::vector<std::vector<std::vector<unsigned char>>> blobs;   // [parity][group]
   bool blobs_valid = false;
+  uint64_t blob_gen = 0;                   // bumped whenever the argument blobs are rebuilt
   void* shell_init_scratch = nullptr;
   std::vector<void*> shell_init_arrays;
   // graph
@@ -215,6 +225,28 @@ struct kf_exec {
 };
 
 namespace kf {
+
+// Renamed array versions that need their own buffer ("redundant arrays"): every version of a
+// relaxed array except the final version of a TEMP array (which lives in the array itself).
+// *period = 2 when a renamed array is step-live (its buffers ping-pong between steps).
+static std::vector<Ver> renamed_versions(const Program& p, int* period) {
+  std::vector<Ver> out;
+  *period = 1;
+  for (int x = 0; x < p.na; x++) {
+    if (!p.relaxed[x]) continue;
+    int w = int(p.writers[x].size());
+    for (int v = 1; v <= w; v++) {
+      if (v == w && !p.step_live[x]) continue;
+      out.push_back(Ver{x, v});
+    }
+    if (p.step_live[x]) *period = 2;
+  }
+  return out;
+}
+
+static uint64_t padded_array_bytes(const Program& p) {
+  return (uint64_t(p.layout.elems) * p.es + 255) / 256 * 256;
+}
 
 static int buffer_id(const kf_exec* E, const Ver& v, int parity) {
   const Program& p = E->prog->p;
@@ -299,6 +331,7 @@ static void build_blobs(kf_exec* E) {
       E->blobs[par][&g - &E->G[0]] = std::move(out);
     }
   E->blobs_valid = true;
+  E->blob_gen++;
 }
 
 // mode 0: every unit; 1: interior tiles only; 2: the other tiles (the group's Split)
@@ -338,7 +371,7 @@ static void run_fill(kf_exec* E, int buf, cudaStream_t s) {
 }
 
 // Consecutive fills of a schedule in one launch (x and y together; z, if periodic, after them).
-static void run_fills(kf_exec* E, const std::vector<int>& bufs, cudaStream_t s) {
+static void run_fills(kf_exec* E, const std::vector<int>& bufs, cudaStream_t s, int zghost = 0) {
   if (bufs.empty()) return;
   const Program& p = E->prog->p;
   Geom gm = geom(p);
@@ -348,7 +381,8 @@ static void run_fills(kf_exec* E, const std::vector<int>& bufs, cudaStream_t s) 
   }
   std::vector<void*> ptr;
   for (int b : bufs) ptr.push_back(buf_ptr(E, b));
-  CK(launch_fill_xy_multi(ptr.data(), int(ptr.size()), p.bc[0] == KF_BC_PERIODIC, p.bc[1] == KF_BC_PERIODIC, p.es, gm, s));
+  CK(launch_fill_xy_multi(ptr.data(), int(ptr.size()), p.bc[0] == KF_BC_PERIODIC, p.bc[1] == KF_BC_PERIODIC, p.es, gm, s,
+                          zghost));
   if (p.bc[2] == KF_BC_PERIODIC)
     for (void* b : ptr) CK(launch_fill(2, b, p.es, gm, s));
 }
@@ -400,10 +434,14 @@ static void ensure_device(kf_exec* E) {
       drv().funcGetAttribute(&g.regs, CU_FUNC_ATTRIBUTE_NUM_REGS, g.fn);
       drv().funcGetAttribute(&g.local, CU_FUNC_ATTRIBUTE_LOCAL_SIZE_BYTES, g.fn);
       // the register cap must not cost local memory (spills): rebuild without it
-      if (g.local > 0 && !g.comp->nocap && g.cg.source.find("__maxnreg__") != std::string::npos)
+      if (g.local > 0 && !g.comp->nocap && g.cg.source.find("__maxnreg__") != std::string::npos) {
         g.comp = compile_nocap(g.cg.source, g.cg.name);
-      else
+        if (drv().moduleUnload) drv().moduleUnload(g.mod);
+        g.mod = nullptr;
+        g.fn = nullptr;
+      } else {
         break;
+      }
     }
   }
   (void)p;
@@ -513,7 +551,14 @@ static void exec_run(kf_exec* E, void* const* arrays, void* scratch, uint64_t sc
     E->shell_init_scratch = scratch;
     E->shell_init_arrays = arr;
   }
-  run_fills(E, E->fill_all, s);
+  // run-start fills: the caller's arrays whole; renamed scratch versions (interior not yet written,
+  // x/y ghosts of interior planes filled after their producer) only on the frozen z ghost planes
+  {
+    std::vector<int> arr_b, scr_b;
+    for (int b : E->fill_all) (b < p.na ? arr_b : scr_b).push_back(b);
+    run_fills(E, arr_b, s);
+    run_fills(E, scr_b, s, p.bc[2] == KF_BC_FROZEN ? 1 : 0);
+  }
   int64_t reps = nsteps / E->period, rem = nsteps % E->period;
   if (E->use_graph && !E->profiling && reps > 0) {
     if (!E->gexec) {
@@ -577,17 +622,8 @@ kf_status kf_exec_create_ex(kf_program* prog, const int32_t* plan, const kf_targ
       fail(KF_E_ILLEGAL_PLAN, "plan violates constraint V" + std::to_string(code) + " in group " + std::to_string(why.group));
     E->order = quotient_order(p, E->plan);
     // renamed versions -> scratch buffers ("redundant arrays")
-    for (int x = 0; x < p.na; x++) {
-      if (!p.relaxed[x]) continue;
-      int w = int(p.writers[x].size());
-      for (int v = 1; v <= w; v++) {
-        if (v == w && !p.step_live[x]) continue;   // final version of a TEMP array lives in the array itself
-        E->scratch_vers.push_back(Ver{x, v});
-      }
-      if (p.step_live[x]) E->period = 2;
-    }
-    E->array_bytes = uint64_t(p.layout.elems) * p.es;
-    E->array_bytes = (E->array_bytes + 255) / 256 * 256;
+    E->scratch_vers = renamed_versions(p, &E->period);
+    E->array_bytes = padded_array_bytes(p);
     E->scratch_bytes = E->array_bytes * E->scratch_vers.size();
     E->G.resize(E->plan.m);
     for (int gi = 0; gi < E->plan.m; gi++) {
@@ -609,8 +645,33 @@ kf_status kf_exec_create_ex(kf_program* prog, const int32_t* plan, const kf_targ
       g.outs = g.L.live_out;
       E->step_bytes += g.bytes;
     }
-    // JIT all groups (NVRTC, sm_100a); identical sources are compiled once per process
-    for (auto& g : E->G) g.comp = compile_cached(g.cg.source, g.cg.name);
+    // JIT all groups (NVRTC, sm_100a) on parallel host threads; identical sources are compiled once
+    // per process (the cache), each nvrtcProgram is private to its thread
+    {
+      const int nthr = std::max(1, std::min<int>(int(E->G.size()), int(std::thread::hardware_concurrency())));
+      std::atomic<int> next{0};
+      std::vector<std::string> errs(E->G.size());
+      std::vector<kf_status> sts(E->G.size(), KF_OK);
+      auto work = [&]() {
+        for (int i = next++; i < int(E->G.size()); i = next++) {
+          try {
+            E->G[i].comp = compile_cached(E->G[i].cg.source, E->G[i].cg.name);
+          } catch (const Error& e) {
+            sts[i] = e.st;
+            errs[i] = e.msg;
+          } catch (const std::exception& e) {
+            sts[i] = KF_E_NVRTC;
+            errs[i] = e.what();
+          }
+        }
+      };
+      std::vector<std::thread> th;
+      for (int t = 1; t < nthr; t++) th.emplace_back(work);
+      work();
+      for (auto& t : th) t.join();
+      for (size_t i = 0; i < sts.size(); i++)
+        if (sts[i] != KF_OK) fail(sts[i], errs[i]);
+    }
     build_schedule(E.get());
     *out = E.release();
   });
@@ -632,6 +693,8 @@ void kf_exec_destroy(kf_exec* ex) {
     for (auto e : ex->evpool) cudaEventDestroy(e);
     for (void* d : ex->dev_arrays) cudaFree(d);
     if (ex->dev_scratch) cudaFree(ex->dev_scratch);
+    for (auto& g : ex->G)
+      if (g.mod && drv().moduleUnload) drv().moduleUnload(g.mod);
   } catch (...) {
   }
   delete ex;
@@ -680,6 +743,9 @@ kf_status kf_run_host(kf_exec* ex, void* const* host_arrays, int64_t nsteps, con
       }
     }
     ex->host_first = false;
+    // the uploaded arrays carry their (FROZEN) ghost values: renamed copies must take them again
+    ex->shell_init_scratch = nullptr;
+    ex->shell_init_arrays.clear();
     exec_run(ex, ex->dev_arrays.data(), ex->dev_scratch, ex->scratch_bytes, nsteps, params, s);
     for (int x = 0; x < p.na; x++)
       if (p.step_live[x]) {
@@ -795,6 +861,14 @@ kf_status kf_exec_group_times(kf_exec* ex, double* ms, int32_t cap, int32_t* n, 
   });
 }
 
+kf_status kf_exec_invalidate(kf_exec* ex) {
+  KF_TRY({
+    if (!ex) fail(KF_E_ARG, "null exec");
+    ex->shell_init_scratch = nullptr;
+    ex->shell_init_arrays.clear();
+  });
+}
+
 kf_status kf_exec_set_graph(kf_exec* ex, int32_t on) {
   KF_TRY({
     if (!ex) fail(KF_E_ARG, "null exec");
@@ -838,9 +912,12 @@ kf_status kf_jit_check(const kf_program* prog, const int32_t* plan, const kf_tar
 // Domain decomposition over a px x py process grid (x, y split; z whole; rank = iy*px + ix).
 // Each part runs the same plan on its local sub-domain; the periodic ghost fills of the
 // single-domain schedule become halo exchanges with the neighbouring parts (x strips first,
-// then y strips including the x ghosts, which covers corners).  Transports: loopback (all
-// parts in one process/GPU, strips copied device-to-device; used to test the decomposition
-// bit-exactly on one GPU) and NCCL send/recv (one process per GPU, NVLink/NVSwitch).
+// then y strips including the x ghosts, which covers corners).  Every exchange point handles all
+// its pending buffers at once: one pack launch, one ncclGroupStart/End of all sends and receives,
+// one unpack launch per phase.  Transports: loopback (all parts in one process/GPU,
+// strips copied device-to-device in one launch per phase; tests the decomposition bit-exactly on
+// one GPU) and NCCL send/recv (one process per GPU, NVLink/NVSwitch).  A replay period of steps
+// is captured in a CUDA graph (exchanges, overlap fork/join and NCCL calls included).
 #include <dlfcn.h>
 
 namespace kf {
@@ -877,7 +954,7 @@ static Nccl& nccl() {
     n.commDestroy = (int (*)(void*))dlsym(h, "ncclCommDestroy");
     n.errStr = (const char* (*)(int))dlsym(h, "ncclGetErrorString");
   });
-  if (!n.h || !n.getUniqueId || !n.commInitRank || !n.send || !n.recv)
+  if (!n.h || !n.getUniqueId || !n.commInitRank || !n.send || !n.recv || !n.groupStart || !n.groupEnd)
     fail(KF_E_UNSUPPORTED, "NCCL (libnccl.so.2) not available");
   return n;
 }
@@ -887,20 +964,45 @@ static void ckn(int r, const char* what) {
   fail(KF_E_NCCL, std::string(what) + ": " + (nccl().errStr ? nccl().errStr(r) : std::to_string(r)));
 }
 
+// One NCCL communicator, shared by the kf_dist objects of one kf_dist_init context.
+struct Comm {
+  void* comm = nullptr;
+  ~Comm() {
+    if (comm && nccl().commDestroy) nccl().commDestroy(comm);
+  }
+};
+
+static std::shared_ptr<Comm> make_comm(int rank, int world, const uint8_t* id) {
+  NcclId u;
+  std::memcpy(&u, id, 128);
+  CK(cudaFree(nullptr));
+  auto c = std::make_shared<Comm>();
+  // ncclCommInitRank(ncclComm_t*, int nranks, ncclUniqueId commId, int rank): id passed by value
+  auto init = (int (*)(void**, int, NcclId, int))nccl().commInitRank;
+  ckn(init(&c->comm, world, u, rank), "ncclCommInitRank");
+  return c;
+}
+
 }  // namespace kf
 
 struct kf_dist {
   std::vector<kf_exec*> parts;   // loopback: px*py parts; NCCL: 1 part
   int px = 1, py = 1, rank = 0, world = 1;
   bool use_nccl = false;
-  void* comm = nullptr;
-  void* stage = nullptr;         // NCCL staging (device): 4 strips of the largest face
-  uint64_t stage_bytes = 0;
+  std::shared_ptr<kf::Comm> comm;
+  void* stage = nullptr;         // NCCL staging (device): 4 strip slots per buffer of a batch
+  uint64_t slot_bytes = 0;       // bytes of one strip slot (the larger face)
+  int max_batch = 1;             // buffers per exchange batch the staging holds
   // overlap (a11): exchanges on a second stream while the group's interior tiles run
   int overlap = 1;
   cudaStream_t xs = nullptr;
   cudaEvent_t ev_ready = nullptr, ev_done = nullptr;
-  int xs_device = -1;
+  // CUDA graph of one replay period
+  bool use_graph = true, graph_failed = false;
+  cudaStream_t cap = nullptr;
+  cudaGraphExec_t gexec = nullptr;
+  std::vector<uint64_t> gens;    // parts' blob generations the graph was captured with
+  int gexec_overlap = -1;
 };
 
 namespace kf {
@@ -922,11 +1024,10 @@ static void strip_boxes(const Program& p, int axis, Box* send_lo, Box* send_hi, 
   const int d = int(p.n[2]) + 2 * p.ghost[2];
   if (axis == 0) {
     const int h = ny + 2 * g1;                    // every row, y ghosts included
-    const long long row0 = 0;
-    *send_lo = Box{row0 + L.xoff, g0, h, d};
-    *send_hi = Box{row0 + L.xoff + nx - g0, g0, h, d};
-    *recv_lo = Box{row0 + L.xoff - g0, g0, h, d};
-    *recv_hi = Box{row0 + L.xoff + nx, g0, h, d};
+    *send_lo = Box{L.xoff, g0, h, d};
+    *send_hi = Box{L.xoff + nx - g0, g0, h, d};
+    *recv_lo = Box{L.xoff - g0, g0, h, d};
+    *recv_hi = Box{L.xoff + nx, g0, h, d};
   } else {
     const int w = int(L.pitch);                   // whole padded rows: x ghosts (and corners) included
     *send_lo = Box{(long long)g1 * L.pitch, w, g1, d};
@@ -936,66 +1037,149 @@ static void strip_boxes(const Program& p, int axis, Box* send_lo, Box* send_hi, 
   }
 }
 
-static void copy_box_buf(const Program& p, void* dst_base, const Box& db, const void* src_base, const Box& sb,
-                         cudaStream_t s) {
-  const kf_layout& L = p.layout;
-  CK(launch_copy_box((char*)dst_base + db.off * p.es, L.pitch, L.plane, (const char*)src_base + sb.off * p.es, L.pitch,
-                     L.plane, sb.w, sb.h, sb.d, p.es, s));
-}
+static uint64_t box_bytes(const Box& b, int es) { return uint64_t(b.w) * b.h * b.d * es; }
 
-// Halo exchange of buffer id `b` on every part: decomposed axes exchange with neighbours,
-// other periodic axes wrap locally.
-static void dist_exchange(kf_dist* D, int b, cudaStream_t s) {
-  const Program& p = D->parts[0]->prog->p;
-  Geom gm = geom(p);
-  for (int axis = 0; axis < 3; axis++) {
-    if (p.bc[axis] != KF_BC_PERIODIC) continue;
-    const int np = axis == 0 ? D->px : (axis == 1 ? D->py : 1);
-    if (np == 1) {
-      for (kf_exec* E : D->parts) CK(launch_fill(axis, buf_ptr(E, b), p.es, gm, s));
-      continue;
-    }
-    Box slo, shi, rlo, rhi;
-    strip_boxes(p, axis, &slo, &shi, &rlo, &rhi);
-    if (!D->use_nccl) {
-      const int nparts = int(D->parts.size());
-      for (int r = 0; r < nparts; r++) {
-        int nb[4];
-        dist_neighbors(D->px, D->py, r, nb);
-        const int lo = axis == 0 ? nb[0] : nb[2], hi = axis == 0 ? nb[1] : nb[3];
-        // my low ghost <- low neighbour's high interior strip; my high ghost <- high neighbour's low strip
-        copy_box_buf(p, buf_ptr(D->parts[r], b), rlo, buf_ptr(D->parts[lo], b), shi, s);
-        copy_box_buf(p, buf_ptr(D->parts[r], b), rhi, buf_ptr(D->parts[hi], b), slo, s);
+// Halo exchange of the buffers `bufs` on every part: decomposed axes exchange with the
+// neighbours, other periodic axes wrap locally.  Batches larger than the staging are split.
+static void dist_exchange(kf_dist* D, const std::vector<int>& all, cudaStream_t s) {
+  if (all.empty()) return;
+  for (size_t c0 = 0; c0 < all.size(); c0 += size_t(D->max_batch)) {
+    const std::vector<int> bufs(all.begin() + c0, all.begin() + std::min(all.size(), c0 + size_t(D->max_batch)));
+    const Program& p = D->parts[0]->prog->p;
+    const Geom gm = geom(p);
+    const int es = p.es;
+    const kf_layout& L = p.layout;
+    for (int axis = 0; axis < 3; axis++) {
+      if (p.bc[axis] != KF_BC_PERIODIC) continue;
+      const int np = axis == 0 ? D->px : (axis == 1 ? D->py : 1);
+      if (np == 1) {
+        if (axis < 2) {
+          std::vector<void*> ptr;
+          for (kf_exec* E : D->parts)
+            for (int b : bufs) ptr.push_back(buf_ptr(E, b));
+          CK(launch_fill_xy_multi(ptr.data(), int(ptr.size()), axis == 0, axis == 1, es, gm, s));
+        } else {
+          for (kf_exec* E : D->parts)
+            for (int b : bufs) CK(launch_fill(2, buf_ptr(E, b), es, gm, s));
+        }
+        continue;
       }
-    } else {
+      Box slo, shi, rlo, rhi;
+      strip_boxes(p, axis, &slo, &shi, &rlo, &rhi);
+      auto at = [&](void* base, const Box& b) { return (void*)((char*)base + b.off * es); };
+      std::vector<BoxCopy> boxes;
+      if (!D->use_nccl) {
+        // my low ghost <- low neighbour's high interior strip; my high ghost <- high neighbour's low strip
+        for (int r = 0; r < int(D->parts.size()); r++) {
+          int nb[4];
+          dist_neighbors(D->px, D->py, r, nb);
+          const int lo = axis == 0 ? nb[0] : nb[2], hi = axis == 0 ? nb[1] : nb[3];
+          for (int b : bufs) {
+            boxes.push_back(BoxCopy{at(buf_ptr(D->parts[r], b), rlo), at(buf_ptr(D->parts[lo], b), shi), L.pitch, L.plane,
+                                    L.pitch, L.plane, shi.w, shi.h, shi.d, 0});
+            boxes.push_back(BoxCopy{at(buf_ptr(D->parts[r], b), rhi), at(buf_ptr(D->parts[hi], b), slo), L.pitch, L.plane,
+                                    L.pitch, L.plane, slo.w, slo.h, slo.d, 0});
+          }
+        }
+        CK(launch_copy_boxes(boxes.data(), int(boxes.size()), es, s));
+        continue;
+      }
       kf_exec* E = D->parts[0];
       int nb[4];
       dist_neighbors(D->px, D->py, D->rank, nb);
       const int lo = axis == 0 ? nb[0] : nb[2], hi = axis == 0 ? nb[1] : nb[3];
-      const uint64_t strip = uint64_t(slo.w) * slo.h * slo.d * p.es;
-      char* st = (char*)D->stage;
-      char *s_lo = st, *s_hi = st + strip, *r_lo = st + 2 * strip, *r_hi = st + 3 * strip;
-      const kf_layout& L = p.layout;
-      auto pack = [&](char* dst, const Box& bx) {
-        CK(launch_copy_box(dst, bx.w, (long long)bx.w * bx.h, (const char*)buf_ptr(E, b) + bx.off * p.es, L.pitch, L.plane,
-                           bx.w, bx.h, bx.d, p.es, s));
-      };
-      auto unpack = [&](const Box& bx, const char* src) {
-        CK(launch_copy_box((char*)buf_ptr(E, b) + bx.off * p.es, L.pitch, L.plane, src, bx.w, (long long)bx.w * bx.h, bx.w,
-                           bx.h, bx.d, p.es, s));
-      };
-      pack(s_lo, slo);
-      pack(s_hi, shi);
+      const uint64_t strip = box_bytes(slo, es);
+      if (strip > D->slot_bytes) fail(KF_E_RESOURCE, "internal: halo strip larger than the staging slot");
+      auto slot = [&](size_t i, int j) { return (char*)D->stage + (4 * i + j) * D->slot_bytes; };   // 0 s_lo 1 s_hi 2 r_lo 3 r_hi
+      // pack the send strips of every buffer (one launch)
+      for (size_t i = 0; i < bufs.size(); i++) {
+        void* base = buf_ptr(E, bufs[i]);
+        boxes.push_back(BoxCopy{slot(i, 0), at(base, slo), slo.w, (long long)slo.w * slo.h, L.pitch, L.plane, slo.w, slo.h, slo.d, 0});
+        boxes.push_back(BoxCopy{slot(i, 1), at(base, shi), shi.w, (long long)shi.w * shi.h, L.pitch, L.plane, shi.w, shi.h, shi.d, 0});
+      }
+      CK(launch_copy_boxes(boxes.data(), int(boxes.size()), es, s));
+      // one group of every send and receive of the phase.  Per peer, the order of matching
+      // operations is the buffer order on both sides: my low strip goes to the low neighbour's
+      // high ghost, which it receives (r_hi) in the same buffer order (also when lo == hi).
       Nccl& n = nccl();
       ckn(n.groupStart(), "ncclGroupStart");
-      ckn(n.send(s_lo, strip, 1 /*ncclUint8*/, lo, D->comm, s), "ncclSend");   // my low strip -> low nbr's high ghost
-      ckn(n.send(s_hi, strip, 1, hi, D->comm, s), "ncclSend");                 // my high strip -> high nbr's low ghost
-      ckn(n.recv(r_hi, strip, 1, hi, D->comm, s), "ncclRecv");                 // high nbr's low strip -> my high ghost
-      ckn(n.recv(r_lo, strip, 1, lo, D->comm, s), "ncclRecv");                 // low nbr's high strip -> my low ghost
+      for (size_t i = 0; i < bufs.size(); i++) {
+        ckn(n.send(slot(i, 0), strip, 1 /*ncclUint8*/, lo, D->comm->comm, s), "ncclSend");
+        ckn(n.send(slot(i, 1), strip, 1, hi, D->comm->comm, s), "ncclSend");
+        ckn(n.recv(slot(i, 3), strip, 1, hi, D->comm->comm, s), "ncclRecv");
+        ckn(n.recv(slot(i, 2), strip, 1, lo, D->comm->comm, s), "ncclRecv");
+      }
       ckn(n.groupEnd(), "ncclGroupEnd");
-      unpack(rlo, r_lo);
-      unpack(rhi, r_hi);
+      boxes.clear();
+      for (size_t i = 0; i < bufs.size(); i++) {
+        void* base = buf_ptr(E, bufs[i]);
+        boxes.push_back(BoxCopy{at(base, rlo), slot(i, 2), L.pitch, L.plane, rlo.w, (long long)rlo.w * rlo.h, rlo.w, rlo.h, rlo.d, 0});
+        boxes.push_back(BoxCopy{at(base, rhi), slot(i, 3), L.pitch, L.plane, rhi.w, (long long)rhi.w * rhi.h, rhi.w, rhi.h, rhi.d, 0});
+      }
+      CK(launch_copy_boxes(boxes.data(), int(boxes.size()), es, s));
     }
+  }
+}
+
+static void profiled_launch(kf_exec* E, int gi, int par, cudaStream_t s) {
+  if (!E->profiling) {
+    launch_group(E, gi, par, s);
+    return;
+  }
+  cudaEvent_t a, b;
+  if (E->evpool.size() >= 2) {
+    a = E->evpool.back(); E->evpool.pop_back();
+    b = E->evpool.back(); E->evpool.pop_back();
+  } else {
+    CK(cudaEventCreate(&a));
+    CK(cudaEventCreate(&b));
+  }
+  CK(cudaEventRecord(a, s));
+  launch_group(E, gi, par, s);
+  CK(cudaEventRecord(b, s));
+  E->pending.emplace_back(gi, a, b);
+  E->launches++;
+}
+
+// One step (schedule parity `par`) of every part: exchanges before the groups that need them.
+static void dist_step(kf_dist* D, int par, cudaStream_t s) {
+  kf_exec* E0 = D->parts[0];
+  const Program& p = E0->prog->p;
+  std::vector<int> pend;   // exchanges due before the next group
+  for (const Op& op : E0->sched_full[par]) {
+    if (op.kind == 0) {
+      pend.push_back(op.buf);
+      continue;
+    }
+    // Overlap: the exchanges run on a second stream, ordered after everything issued
+    // so far, while the group's interior tiles -- at least one ghost width inside the local domain
+    // in x and y, so they read no x/y ghost and write no strip an exchange packs -- run on the
+    // compute stream; the remaining tiles wait for the exchanges.  Not with a periodic z axis: its
+    // wrap rewrites the z ghost planes, which interior tiles read.
+    const bool split = D->overlap && !pend.empty() && E0->G[op.group].split.ok && !E0->profiling &&
+                       p.bc[2] != KF_BC_PERIODIC;
+    if (split) {
+      CK(cudaEventRecord(D->ev_ready, s));
+      CK(cudaStreamWaitEvent(D->xs, D->ev_ready, 0));
+      dist_exchange(D, pend, D->xs);
+      CK(cudaEventRecord(D->ev_done, D->xs));
+      for (kf_exec* E : D->parts) launch_group(E, op.group, par, s, 1);
+      CK(cudaStreamWaitEvent(s, D->ev_done, 0));
+      for (kf_exec* E : D->parts) launch_group(E, op.group, par, s, 2);
+      pend.clear();
+      continue;
+    }
+    dist_exchange(D, pend, s);
+    pend.clear();
+    for (kf_exec* E : D->parts) profiled_launch(E, op.group, par, s);
+  }
+  dist_exchange(D, pend, s);
+}
+
+static void dist_invalidate_graph(kf_dist* D) {
+  if (D->gexec) {
+    cudaGraphExecDestroy(D->gexec);
+    D->gexec = nullptr;
   }
 }
 
@@ -1004,6 +1188,7 @@ static void dist_run(kf_dist* D, void* const* arrays, void* const* scratch, uint
   const Program& p = D->parts[0]->prog->p;
   const int np = int(D->parts.size());
   if (!arrays) fail(KF_E_ARG, "arrays is NULL");
+  if (p.n_params > 0 && !params) fail(KF_E_ARG, "params is NULL but the program has PARAM slots");
   for (int r = 0; r < np; r++) {
     kf_exec* E = D->parts[r];
     void* const* arr = arrays + size_t(r) * p.na;
@@ -1024,63 +1209,56 @@ static void dist_run(kf_dist* D, void* const* arrays, void* const* scratch, uint
     }
   }
   kf_exec* E0 = D->parts[0];
-  for (int b : E0->fill_all) dist_exchange(D, b, s);
-  if (D->overlap && !D->xs) {
-    CK(cudaGetDevice(&D->xs_device));
+  dist_exchange(D, E0->fill_all, s);
+  if (!D->xs) {
     CK(cudaStreamCreateWithFlags(&D->xs, cudaStreamNonBlocking));
     CK(cudaEventCreateWithFlags(&D->ev_ready, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&D->ev_done, cudaEventDisableTiming));
   }
-  std::vector<int> pend;   // exchanges due before the next group
-  for (int64_t step = 0; step < nsteps; step++) {
-    const int par = int(step % E0->period);
-    for (const Op& op : E0->sched_full[par]) {
-      if (op.kind == 0) {
-        pend.push_back(op.buf);
-        continue;
+  bool profiling = false;
+  std::vector<uint64_t> gens;
+  for (kf_exec* E : D->parts) {
+    profiling = profiling || E->profiling;
+    gens.push_back(E->blob_gen);
+  }
+  const int64_t reps = nsteps / E0->period, rem = nsteps % E0->period;
+  bool done = false;
+  if (D->use_graph && !D->graph_failed && !profiling && reps > 0) {
+    if (D->gexec && (gens != D->gens || D->gexec_overlap != D->overlap)) dist_invalidate_graph(D);
+    if (!D->gexec) {
+      if (!D->cap) CK(cudaStreamCreateWithFlags(&D->cap, cudaStreamNonBlocking));
+      cudaGraph_t graph = nullptr;
+      CK(cudaStreamBeginCapture(D->cap, cudaStreamCaptureModeThreadLocal));
+      try {
+        for (int par = 0; par < E0->period; par++) dist_step(D, par, D->cap);
+      } catch (...) {
+        cudaStreamEndCapture(D->cap, &graph);
+        if (graph) cudaGraphDestroy(graph);
+        cudaGetLastError();
+        throw;
       }
-      // Overlap: the exchanges run on a second stream, ordered after everything
-      // issued so far, while the group's interior tiles -- at least one ghost width inside the
-      // local domain, so they read no ghost and write no strip an exchange packs -- run on the
-      // compute stream; the remaining tiles wait for the exchanges.
-      const bool split = D->overlap && !pend.empty() && E0->G[op.group].split.ok && !E0->profiling;
-      if (split) {
-        CK(cudaEventRecord(D->ev_ready, s));
-        CK(cudaStreamWaitEvent(D->xs, D->ev_ready, 0));
-        for (int b : pend) dist_exchange(D, b, D->xs);
-        CK(cudaEventRecord(D->ev_done, D->xs));
-        for (kf_exec* E : D->parts) launch_group(E, op.group, par, s, 1);
-        CK(cudaStreamWaitEvent(s, D->ev_done, 0));
-        for (kf_exec* E : D->parts) launch_group(E, op.group, par, s, 2);
-        pend.clear();
-        continue;
-      }
-      for (int b : pend) dist_exchange(D, b, s);
-      pend.clear();
-      {
-        for (kf_exec* E : D->parts) {
-          if (!E->profiling) {
-            launch_group(E, op.group, par, s);
-            continue;
-          }
-          cudaEvent_t a, b;
-          if (E->evpool.size() >= 2) {
-            a = E->evpool.back(); E->evpool.pop_back();
-            b = E->evpool.back(); E->evpool.pop_back();
-          } else {
-            CK(cudaEventCreate(&a));
-            CK(cudaEventCreate(&b));
-          }
-          CK(cudaEventRecord(a, s));
-          launch_group(E, op.group, par, s);
-          CK(cudaEventRecord(b, s));
-          E->pending.emplace_back(op.group, a, b);
-          E->launches++;
-        }
+      cudaError_t e = cudaStreamEndCapture(D->cap, &graph);
+      if (e == cudaSuccess && graph) e = cudaGraphInstantiate(&D->gexec, graph, 0);
+      if (graph) cudaGraphDestroy(graph);
+      if (e != cudaSuccess) {   // e.g. a transport that cannot be captured: run eagerly from now on
+        cudaGetLastError();
+        D->gexec = nullptr;
+        D->graph_failed = true;
+      } else {
+        D->gens = gens;
+        D->gexec_overlap = D->overlap;
       }
     }
+    if (D->gexec) {
+      // the graph's first node must follow the stream's earlier work (ghost exchanges above)
+      for (int64_t r = 0; r < reps; r++) CK(cudaGraphLaunch(D->gexec, s));
+      done = true;
+    }
   }
-  for (int b : pend) dist_exchange(D, b, s);
+  if (!done)
+    for (int64_t r = 0; r < reps; r++)
+      for (int par = 0; par < E0->period; par++) dist_step(D, par, s);
+  for (int64_t r = 0; r < rem; r++) dist_step(D, int(r), s);
   if (E0->period == 2 && (nsteps % 2) == 1)
     for (kf_exec* E : D->parts)
       for (int x = 0; x < p.na; x++)
@@ -1089,6 +1267,96 @@ static void dist_run(kf_dist* D, void* const* arrays, void* const* scratch, uint
           CK(cudaMemcpyAsync(E->cur_arrays[x], buf_ptr(E, b), E->array_bytes, cudaMemcpyDeviceToDevice, s));
         }
   CK(cudaGetLastError());
+}
+
+// Builds a kf_dist over parts (loopback when comm is null and n_parts == px*py; NCCL otherwise).
+static kf_dist* dist_make(kf_exec* const* parts, int n_parts, int px, int py, int rank, int world,
+                          std::shared_ptr<Comm> comm) {
+  if (!parts || n_parts < 1 || px < 1 || py < 1) fail(KF_E_ARG, "bad arguments");
+  auto D = std::make_unique<kf_dist>();
+  D->px = px;
+  D->py = py;
+  D->rank = rank;
+  D->world = world;
+  for (int i = 0; i < n_parts; i++) {
+    if (!parts[i]) fail(KF_E_ARG, "null part");
+    D->parts.push_back(parts[i]);
+  }
+  const Program& p = parts[0]->prog->p;
+  for (int i = 1; i < n_parts; i++)
+    if (parts[i]->prog != parts[0]->prog || parts[i]->plan.label != parts[0]->plan.label)
+      fail(KF_E_ARG, "all parts must run the same program and plan");
+  if ((px > 1 && p.bc[0] != KF_BC_PERIODIC) || (py > 1 && p.bc[1] != KF_BC_PERIODIC))
+    fail(KF_E_UNSUPPORTED, "decomposed axes must be PERIODIC in the local program (halo exchange replaces the wrap)");
+  if ((px > 1 && p.n[0] < p.ghost[0]) || (py > 1 && p.n[1] < p.ghost[1]))
+    fail(KF_E_ARG, "local extent smaller than the ghost width");
+  // the largest batch of buffers one exchange point handles (the schedule's, and the run-start fills)
+  int batch = 1, run = 0;
+  for (auto& ops : parts[0]->sched_full) {
+    for (const Op& op : ops) {
+      if (op.kind == 0) batch = std::max(batch, ++run);
+      else run = 0;
+    }
+    run = 0;
+  }
+  D->max_batch = std::max(batch, 1);
+  if (n_parts == px * py && world == 1 && !comm) {
+    D->use_nccl = false;   // loopback: every part in this process
+  } else if (n_parts == 1 && world == px * py && rank >= 0 && rank < world && comm) {
+    D->use_nccl = true;
+    D->comm = comm;
+    Box a, b, c, d;
+    strip_boxes(p, 0, &a, &b, &c, &d);
+    uint64_t fx = box_bytes(a, p.es);
+    strip_boxes(p, 1, &a, &b, &c, &d);
+    uint64_t fy = box_bytes(a, p.es);
+    D->slot_bytes = (std::max(fx, fy) + 255) / 256 * 256;
+    const uint64_t bytes = 4 * D->slot_bytes * uint64_t(D->max_batch);
+    if (cudaMalloc(&D->stage, bytes) != cudaSuccess) fail(KF_E_OOM, "cudaMalloc (halo staging) failed");
+  } else {
+    fail(KF_E_ARG, "either n_parts == px*py with world == 1 (loopback) or n_parts == 1 with world == px*py (NCCL)");
+  }
+  return D.release();
+}
+
+static void dist_free(kf_dist* d) {
+  if (!d) return;
+  try {
+    dist_invalidate_graph(d);
+    if (d->cap) cudaStreamDestroy(d->cap);
+    if (d->stage) cudaFree(d->stage);
+    if (d->xs) cudaStreamDestroy(d->xs);
+    if (d->ev_ready) cudaEventDestroy(d->ev_ready);
+    if (d->ev_done) cudaEventDestroy(d->ev_done);
+  } catch (...) {
+  }
+  delete d;
+}
+
+// ---------------------------------------------------------------- kf_run (§8(b) entry point)
+// Per-program cache of executors by canonical plan (JIT once per plan and device), plus the
+// distributed context of kf_dist_init.
+struct RunCache {
+  std::map<std::pair<int, std::vector<int>>, kf_exec*> execs;   // (device, canonical plan)
+  std::map<kf_exec*, kf_dist*> dists;
+  bool dist = false;
+  int rank = 0, world = 1, px = 1, py = 1;
+  std::shared_ptr<Comm> comm;
+};
+
+static void run_cache_free(void* v) {
+  RunCache* c = static_cast<RunCache*>(v);
+  for (auto& [e, d] : c->dists) dist_free(d);
+  for (auto& [k, e] : c->execs) kf_exec_destroy(e);
+  delete c;
+}
+
+static RunCache& run_cache(kf_program* prog) {
+  if (!prog->run_cache) {
+    prog->run_cache = new RunCache();
+    prog->run_cache_free = run_cache_free;
+  }
+  return *static_cast<RunCache*>(prog->run_cache);
 }
 
 }  // namespace kf
@@ -1113,47 +1381,28 @@ kf_status kf_dist_neighbors(int32_t px, int32_t py, int32_t rank, int32_t out[4]
   });
 }
 
+kf_status kf_dist_strips(const kf_program* prog, int32_t axis, kf_box out[4]) {
+  KF_TRY({
+    if (!prog || !out) fail(KF_E_ARG, "null argument");
+    if (axis < 0 || axis > 1) fail(KF_E_ARG, "axis must be 0 (x) or 1 (y)");
+    Box b[4];
+    strip_boxes(prog->p, axis, &b[0], &b[1], &b[2], &b[3]);
+    for (int i = 0; i < 4; i++) out[i] = kf_box{b[i].off, b[i].w, b[i].h, b[i].d, 0};
+  });
+}
+
 kf_status kf_dist_create(kf_exec* const* parts, int32_t n_parts, int32_t px, int32_t py, int32_t rank, int32_t world,
                          const uint8_t* nccl_id, kf_dist** out) {
   KF_TRY({
-    if (!parts || !out || n_parts < 1 || px < 1 || py < 1) fail(KF_E_ARG, "bad arguments");
-    auto D = std::make_unique<kf_dist>();
-    D->px = px;
-    D->py = py;
-    D->rank = rank;
-    D->world = world;
-    for (int i = 0; i < n_parts; i++) {
-      if (!parts[i]) fail(KF_E_ARG, "null part");
-      D->parts.push_back(parts[i]);
-    }
-    const Program& p = parts[0]->prog->p;
-    for (int i = 1; i < n_parts; i++)
-      if (parts[i]->prog != parts[0]->prog || parts[i]->plan.label != parts[0]->plan.label)
-        fail(KF_E_ARG, "all parts must run the same program and plan");
-    if ((px > 1 && p.bc[0] != KF_BC_PERIODIC) || (py > 1 && p.bc[1] != KF_BC_PERIODIC))
-      fail(KF_E_UNSUPPORTED, "decomposed axes must be PERIODIC in the local program (halo exchange replaces the wrap)");
-    if ((px > 1 && p.n[0] < p.ghost[0]) || (py > 1 && p.n[1] < p.ghost[1]))
-      fail(KF_E_ARG, "local extent smaller than the ghost width");
-    if (n_parts == px * py && world == 1) {
-      D->use_nccl = false;   // loopback: every part in this process
-    } else if (n_parts == 1 && world == px * py && rank >= 0 && rank < world) {
+    if (!out) fail(KF_E_ARG, "null argument");
+    std::shared_ptr<Comm> comm;
+    if (!(n_parts == px * py && world == 1)) {
       if (!nccl_id) fail(KF_E_ARG, "nccl_id required for the NCCL transport");
-      D->use_nccl = true;
-      NcclId u;
-      std::memcpy(&u, nccl_id, 128);
-      CK(cudaFree(nullptr));
-      // ncclCommInitRank(ncclComm_t*, int nranks, ncclUniqueId commId, int rank): id passed by value
-      auto init = (int (*)(void**, int, NcclId, int))nccl().commInitRank;
-      ckn(init(&D->comm, world, u, rank), "ncclCommInitRank");
-      const kf_layout& L = p.layout;
-      uint64_t fx = uint64_t(p.ghost[0]) * (p.n[1] + 2 * p.ghost[1]) * (p.n[2] + 2 * p.ghost[2]);
-      uint64_t fy = uint64_t(L.pitch) * p.ghost[1] * (p.n[2] + 2 * p.ghost[2]);
-      D->stage_bytes = 4 * std::max(fx, fy) * p.es;
-      if (cudaMalloc(&D->stage, D->stage_bytes) != cudaSuccess) fail(KF_E_OOM, "cudaMalloc (halo staging) failed");
-    } else {
-      fail(KF_E_ARG, "either n_parts == px*py with world == 1 (loopback) or n_parts == 1 with world == px*py (NCCL)");
+      if (n_parts != 1 || world != px * py || rank < 0 || rank >= world)
+        fail(KF_E_ARG, "either n_parts == px*py with world == 1 (loopback) or n_parts == 1 with world == px*py (NCCL)");
+      comm = make_comm(rank, world, nccl_id);
     }
-    *out = D.release();
+    *out = dist_make(parts, n_parts, px, py, rank, world, comm);
   });
 }
 
@@ -1173,17 +1422,80 @@ kf_status kf_dist_set_overlap(kf_dist* d, int32_t on) {
   });
 }
 
-void kf_dist_destroy(kf_dist* d) {
-  if (!d) return;
-  try {
-    if (d->comm && nccl().commDestroy) nccl().commDestroy(d->comm);
-    if (d->stage) cudaFree(d->stage);
-    if (d->xs) cudaStreamDestroy(d->xs);
-    if (d->ev_ready) cudaEventDestroy(d->ev_ready);
-    if (d->ev_done) cudaEventDestroy(d->ev_done);
-  } catch (...) {
-  }
-  delete d;
+kf_status kf_dist_set_graph(kf_dist* d, int32_t on) {
+  KF_TRY({
+    if (!d) fail(KF_E_ARG, "null dist");
+    d->use_graph = on != 0;
+    if (!d->use_graph) dist_invalidate_graph(d);
+  });
+}
+
+void kf_dist_destroy(kf_dist* d) { dist_free(d); }
+
+kf_status kf_dist_init(kf_program* prog, int32_t rank, int32_t world, int32_t px, int32_t py, const uint8_t id[128]) {
+  KF_TRY({
+    if (!prog) fail(KF_E_ARG, "null program");
+    if (px < 1 || py < 1 || world != px * py || rank < 0 || rank >= world) fail(KF_E_ARG, "bad process grid or rank");
+    const Program& p = prog->p;
+    if ((px > 1 && p.bc[0] != KF_BC_PERIODIC) || (py > 1 && p.bc[1] != KF_BC_PERIODIC))
+      fail(KF_E_UNSUPPORTED, "decomposed axes must be PERIODIC in the local program");
+    RunCache& c = run_cache(prog);
+    if (c.dist) fail(KF_E_ARG, "kf_dist_init already called for this program");
+    std::shared_ptr<Comm> comm;
+    if (world > 1) {
+      if (!id) fail(KF_E_ARG, "id required when world > 1");
+      comm = make_comm(rank, world, id);
+    }
+    c.dist = world > 1;
+    c.rank = rank;
+    c.world = world;
+    c.px = px;
+    c.py = py;
+    c.comm = comm;
+  });
+}
+
+kf_status kf_scratch_bytes(const kf_program* prog, const int32_t* plan, uint64_t* bytes) {
+  KF_TRY({
+    if (!prog || !bytes) fail(KF_E_ARG, "null argument");
+    (void)plan;   // renamed versions depend on the program only, not on the plan
+    int period = 1;
+    *bytes = padded_array_bytes(prog->p) * renamed_versions(prog->p, &period).size();
+  });
+}
+
+kf_status kf_run(kf_program* prog, const int32_t* plan, void* const* arrays, void* scratch, uint64_t scratch_bytes,
+                 int64_t nsteps, const double* params, void* cuda_stream) {
+  KF_TRY({
+    if (!prog || !plan) fail(KF_E_ARG, "null argument");
+    const Program& p = prog->p;
+    for (int k = 0; k < p.nk; k++)
+      if (plan[k] < 0) fail(KF_E_ILLEGAL_PLAN, "V1 PARTITION: kernel " + std::to_string(k) + " has no group");
+    const Plan pl = make_plan(p, plan);
+    int dev = 0;
+    CK(cudaGetDevice(&dev));
+    RunCache& c = run_cache(prog);
+    auto key = std::make_pair(dev, pl.label);
+    auto it = c.execs.find(key);
+    if (it == c.execs.end()) {
+      kf_target t;
+      kf_target_b200(&t);
+      if (c.dist) t.internal_axes = (c.px > 1 ? 1 : 0) | (c.py > 1 ? 2 : 0);
+      kf_exec* e = nullptr;
+      kf_status st = kf_exec_create(prog, pl.label.data(), &t, &e);
+      if (st != KF_OK) fail(st, kf_last_error());
+      it = c.execs.emplace(key, e).first;
+    }
+    kf_exec* E = it->second;
+    if (!c.dist) {
+      exec_run(E, arrays, scratch, scratch_bytes, nsteps, params, (cudaStream_t)cuda_stream);
+      return KF_OK;
+    }
+    auto dit = c.dists.find(E);
+    if (dit == c.dists.end()) dit = c.dists.emplace(E, dist_make(&E, 1, c.px, c.py, c.rank, c.world, c.comm)).first;
+    void* sc[1] = {scratch};
+    dist_run(dit->second, arrays, sc, scratch_bytes, nsteps, params, (cudaStream_t)cuda_stream);
+  });
 }
 
 }  // extern "C"

@@ -446,4 +446,22 @@ kf_status kf_plan_count_legal(const kf_program* prog, const kf_target* target, u
   });
 }
 
+kf_status kf_plan_enumerate(const kf_program* prog, const kf_target* target, int32_t* plans, int64_t cap,
+                            int64_t* count) {
+  KF_TRY({
+    if (!prog || !count || (cap > 0 && !plans)) fail(KF_E_ARG, "null argument");
+    check_target(target);
+    const Program& p = prog->p;
+    if (p.nk > 14) fail(KF_E_UNSUPPORTED, "enumeration limited to 14 kernels");
+    Evaluator ev(p, *target);
+    int64_t c = 0;
+    enumerate(p, [&](const std::vector<int>& lab, int m) {
+      if (!ev.legal(lab, m, nullptr)) return;
+      if (c < cap) std::copy(lab.begin(), lab.end(), plans + c * p.nk);
+      c++;
+    });
+    *count = c;
+  });
+}
+
 }  // extern "C"

@@ -255,3 +255,59 @@ def test_codegen_pair_canvas_and_split_compile_for_sm100a():
         for kw in (dict(pblock=(2, 1)), dict(pblock=(2, 1), canvas_ld=0, pair_zq=0)):
             regs, spill, log = p.jit_check(plan, g, kf.Target(tile=(32, 8, 0), **kw))
             assert "sm_100a" in log and spill == 0, (g, kw, spill)
+
+
+def test_north_star_entry_points_exported():
+    """SURVEY 8(b) names (P:238 problem statement): kf_run, kf_scratch_bytes, kf_dist_init,
+    kf_program_array_class next to the executor-level calls."""
+    syms = header_symbols()
+    for s in ("kf_program_create", "kf_plan_validate", "kf_project", "kf_run", "kf_scratch_bytes", "kf_dist_init",
+              "kf_dist_unique_id", "kf_program_array_class", "kf_program_edges", "kf_array_layout", "kf_plan_search"):
+        assert s in syms, s
+
+
+@pytest.mark.parametrize("flags", [0, PROG_RELAX_EXPANDABLE, PROG_RELAX_ALL])
+def test_array_classes_and_scratch_bytes(flags):
+    desc = P.weather(n=(24, 16, 6)).with_(flags=flags)
+    p = kf.Program(desc)
+    assert p.array_classes() == [G.array_class(desc, x) for x in range(len(desc.arrays))]
+    # one buffer per renamed version (P:53) except the final version of a TEMP array
+    L_ = p.layout()
+    es = 8
+    per = (L_.elems * es + 255) // 256 * 256
+    nver = 0
+    for x in range(len(desc.arrays)):
+        if G.relaxed(desc, x):
+            w = len(G.writers(desc, x))
+            nver += w if G.step_live(desc, x) else w - 1
+    assert p.scratch_bytes() == per * nver
+    assert p.scratch_bytes([0] * len(desc.kernels)) == per * nver
+
+
+@pytest.mark.parametrize("n,ghost", [((24, 16, 6), (2, 2, 2)), ((17, 9, 5), (3, 2, 2))])
+def test_dist_strip_geometry(n, ghost):
+    """kf_dist_strips: send strips are the first/last ghost-deep interior columns (x) or rows (y,
+    whole padded rows); receive strips are the ghost layers next to them."""
+    from workloads.program import BC_PERIODIC as PER
+    desc = P.weather(n=n, ghost=ghost).with_(bc=(PER, PER, BC_FROZEN))
+    p = kf.Program(desc)
+    L_ = p.layout()
+    gx, gy, gz = ghost
+    nx, ny, nz = n
+    d = nz + 2 * gz
+    sx = p.dist_strips(0)
+    assert sx == [(L_.xoff, gx, ny + 2 * gy, d), (L_.xoff + nx - gx, gx, ny + 2 * gy, d),
+                  (L_.xoff - gx, gx, ny + 2 * gy, d), (L_.xoff + nx, gx, ny + 2 * gy, d)]
+    sy = p.dist_strips(1)
+    assert sy == [(gy * L_.pitch, L_.pitch, gy, d), (ny * L_.pitch, L_.pitch, gy, d),
+                  (0, L_.pitch, gy, d), ((gy + ny) * L_.pitch, L_.pitch, gy, d)]
+
+
+@pytest.mark.parametrize("which", ["tiny", "fig3", "random"])
+def test_plan_enumerate_equals_oracle_legal_set(which):
+    desc = {"tiny": P.tiny(), "fig3": P.fig3(), "random": P.random_program(77, nk=6, na=5)}[which]
+    p = kf.Program(desc)
+    got = sorted(tuple(x) for x in p.legal_plans())
+    ref = sorted(tuple(x) for x in En.legal_plans(desc))
+    assert got == ref
+    assert len(got) == p.count_legal()

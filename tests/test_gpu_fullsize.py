@@ -6,9 +6,9 @@ import numpy as np
 import pytest
 
 from oracle import interp
+from oracle.windows import crop, dependency_radius
 from workloads import data as D
 from workloads import programs as P
-from workloads.program import BC_FROZEN
 
 from .gpu_util import bits
 
@@ -18,29 +18,6 @@ if not torch.cuda.is_available():
     pytest.skip("needs a GPU", allow_module_level=True)
 
 import paper_conf_sc_wahibm14_b200 as kf  # noqa: E402
-
-
-def dependency_radius(desc, nsteps):
-    """xy radius of the cone through which an output after `nsteps` depends on the inputs."""
-    rad = {x: 0 for x in range(len(desc.arrays))}
-    for _ in range(nsteps):
-        for kern in desc.kernels:
-            r = max(rad[a] + max(max(abs(d[0]), abs(d[1])) for d in offs) for a, offs in kern.reads().items())
-            for o in kern.writes():
-                rad[o] = max(rad[o], r)
-    return max(rad.values())
-
-
-def crop(desc, arrays, x0, y0, w, margin):
-    """Window [x0, x0+w) x [y0, y0+w) plus margin, wrapped on the periodic xy axes, as a frozen-xy
-    sub-problem (its ghost cells are the true neighbours)."""
-    nx, ny, nz = desc.n
-    g = desc.ghost
-    W = w + 2 * margin
-    xi = (np.arange(-margin - g[0], w + margin + g[0]) + x0) % nx + g[0]
-    yi = (np.arange(-margin - g[1], w + margin + g[1]) + y0) % ny + g[1]
-    sub = desc.with_(n=(W, W, nz), bc=(BC_FROZEN, BC_FROZEN, desc.bc[2]))
-    return sub, {nm: np.ascontiguousarray(a[:, yi][:, :, xi]) for nm, a in arrays.items()}
 
 
 def test_weather_full_size_sampled_windows():
@@ -74,21 +51,25 @@ def test_weather_full_size_sampled_windows():
 
 
 def test_weather_full_size_bench_configuration():
-    """The exact configuration of the committed bench line (profiles/round1_s3_bench_final.json:
-    its plan labels and autotuned per-group launch configurations -- canvas pairs, z register
-    queues, unpredicated loads, TMA stages, z chunks), at full size, on sampled windows."""
+    """The exact configuration of the committed bench line (profiles/bench_timed_config.json,
+    refreshed with every committed bench: its plan labels and autotuned per-group launch
+    configurations -- canvas pairs, z register queues, unpredicated loads, TMA stages, z chunks,
+    ghost writes), at full size, on sampled windows."""
     import json
     import os
-    line = json.load(open(os.path.join(os.path.dirname(__file__), "..", "profiles", "round1_s3_bench_final.json")))
-    plan = line["config"]["plan_labels"]
-    tuned = line["config"]["per_group_launch_config"]
+    line = json.load(open(os.path.join(os.path.dirname(__file__), "..", "profiles", "bench_timed_config.json")))
+    plan = line["plan_labels"]
+    tuned = line["per_group_launch_config"]
+    gw = line.get("ghostwrite", 0)
     desc = P.weather(n=(512, 512, 128))
     inputs = D.weather_inputs(desc, 3)
     prog = kf.Program(desc)
     gt = [kf.Target(tile=tuple(c[0]), stages=c[1], zunroll=c[2], ringunroll=c[3], minblocks=c[4], canvas_ld=c[5],
-                    pblock=(c[6], 1), pair_zq=c[7]) for c in tuned]
+                    pblock=(c[6], 1), pair_zq=c[7], ghostwrite=gw) for c in tuned]
     nsteps = 2
     ex = kf.Exec(prog, plan, kf.Target(tile=(32, 8, 64)), group_targets=gt)
+    if gw:
+        assert ex.info().fills_per_step == 0
     dev = kf.device_arrays(prog, inputs)
     sb = ex.scratch_bytes()
     scr = torch.empty(sb, dtype=torch.uint8, device="cuda") if sb else None
@@ -99,7 +80,7 @@ def test_weather_full_size_bench_configuration():
     M = dependency_radius(desc, nsteps) + 1
     w = 8
     g = desc.ghost
-    for (x0, y0) in ((0, 0), (508, 3), (200, 505), (131, 257), (64, 64)):
+    for (x0, y0) in ((0, 0), (508, 3), (200, 505), (131, 257), (64, 64), (504, 504)):
         sub, sin = crop(desc, inputs, x0, y0, w, M)
         ref = interp.run(sub, sin, nsteps)
         for nm in ("DENS", "MOMX", "MOMY", "MOMZ", "RHOT"):
