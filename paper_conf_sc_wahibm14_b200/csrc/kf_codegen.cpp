@@ -144,7 +144,9 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
   // register cap (__maxnreg__): at most what keeps the shared-memory-limited number of CTAs per SM
   // resident (minblocks 0; or minblocks CTAs) and never above the resource model's estimate R_est
   // (V8, R20).  The runtime recompiles without the cap if it would make ptxas spill.
-  if (L.minblocks >= 0) {
+  if (const char* fc = getenv("KF_MAXNREG")) {   // experiments only: force a register cap
+    o << "#define KF_BOUNDS __maxnreg__(" << atoi(fc) << ")\n";
+  } else if (L.minblocks >= 0) {
     const int smem_ctas = 233472 / std::max(1, L.smem + 1024);
     const int minb = L.minblocks > 0 ? L.minblocks : std::max(1, std::min({smem_ctas, 2048 / std::max(1, NT), 8}));
     const int cap = std::max(24, std::min({65536 / (NT * minb) / 8 * 8, L.regs, 255}));
@@ -569,24 +571,6 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
           const int oi = out_index(Ver{K.stmts[si].out, p.vw(k, K.stmts[si].out)});
           if (oi >= 0) o << "        a.out[" << oi << "][gi] = " << vals[si] << ";\n";
         }
-        if (L.ghost_write) {
-          const std::string gx = "cgx" + rs, gy = "cgy" + rs;
-          o << "        if (edge_tile) {\n";
-          o << "          const bool wx = " << (p.bc[0] == KF_BC_PERIODIC ? "(" + gx + " < GX || " + gx + " >= NX - GX)" : "false")
-            << ", wy = " << (p.bc[1] == KF_BC_PERIODIC ? "(" + gy + " < GY || " + gy + " >= NY - GY)" : "false") << ";\n";
-          o << "          if (wx || wy) {\n";
-          o << "            const int gx2 = " << gx << " < GX ? " << gx << " + NX : " << gx << " - NX;\n";
-          o << "            const int gy2 = " << gy << " < GY ? " << gy << " + NY : " << gy << " - NY;\n";
-          o << "            const long long pb = (long long)" << pz << " * PLANE;\n";
-          for (size_t si = 0; si < K.stmts.size(); si++) {
-            const int oi = out_index(Ver{K.stmts[si].out, p.vw(k, K.stmts[si].out)});
-            if (oi < 0) continue;
-            o << "            if (wx) a.out[" << oi << "][pb + (long long)" << gy << " * PITCH + gx2] = " << vals[si] << ";\n";
-            o << "            if (wy) a.out[" << oi << "][pb + (long long)gy2 * PITCH + " << gx << "] = " << vals[si] << ";\n";
-            o << "            if (wx && wy) a.out[" << oi << "][pb + (long long)gy2 * PITCH + gx2] = " << vals[si] << ";\n";
-          }
-          o << "          }\n        }\n";
-        }
         o << "      }\n";
       }
     }
@@ -854,38 +838,6 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
         for (size_t si = 0; si < K.stmts.size(); si++) {
           const int oi = out_index(Ver{K.stmts[si].out, p.vw(k, K.stmts[si].out)});
           if (oi >= 0) o << "        *(real2*)&a.out[" << oi << "][gi] = real2{" << v0[si] << ", " << v1[si] << "};\n";
-        }
-        if (L.ghost_write) {
-          // periodic x/y ghost copies of the pair (edge tiles only): a y ghost row takes the pair as a
-          // vector (same x); x ghosts and corners point by point (the ghost width may be odd)
-          const bool px_ = p.bc[0] == KF_BC_PERIODIC, py_ = p.bc[1] == KF_BC_PERIODIC;
-          o << "        if (edge_tile) {\n";
-          o << "          const long long pb = (long long)" << pz << " * PLANE;\n";
-          o << "          const bool wy = " << (py_ ? "(cgy_r0 < GY || cgy_r0 >= NY - GY)" : "false") << ";\n";
-          o << "          const int gy2 = cgy_r0 < GY ? cgy_r0 + NY : cgy_r0 - NY;\n";
-          o << "          if (wy) {\n";
-          for (size_t si = 0; si < K.stmts.size(); si++) {
-            const int oi = out_index(Ver{K.stmts[si].out, p.vw(k, K.stmts[si].out)});
-            if (oi >= 0)
-              o << "            *(real2*)&a.out[" << oi << "][pb + (long long)gy2 * PITCH + cgx_r0] = real2{" << v0[si] << ", "
-                << v1[si] << "};\n";
-          }
-          o << "          }\n";
-          if (px_)
-            for (int j = 0; j < 2; j++) {
-              o << "          { const int gxj = cgx_r0 + " << j << ";\n";
-              o << "            if (gxj < GX || gxj >= NX - GX) {\n";
-              o << "              const int gx2 = gxj < GX ? gxj + NX : gxj - NX;\n";
-              for (size_t si = 0; si < K.stmts.size(); si++) {
-                const int oi = out_index(Ver{K.stmts[si].out, p.vw(k, K.stmts[si].out)});
-                if (oi < 0) continue;
-                const std::string& v = j ? v1[si] : v0[si];
-                o << "              a.out[" << oi << "][pb + (long long)cgy_r0 * PITCH + gx2] = " << v << ";\n";
-                o << "              if (wy) a.out[" << oi << "][pb + (long long)gy2 * PITCH + gx2] = " << v << ";\n";
-              }
-              o << "            }\n          }\n";
-            }
-          o << "        }\n";
         }
         o << "      }\n";
       }
@@ -1158,26 +1110,6 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
           << ";\n";
         for (auto& oi : outs)
           if (oi.outi >= 0) o << ind << "  a.out[" << oi.outi << "][gi] = " << vals[oi.stmt] << ";\n";
-        if (L.ghost_write) {
-          // periodic x/y: points within the ghost width of a boundary are also written to the
-          // opposite ghost layer (and corners), so later groups read wrapped halos without fills
-          const std::string gx = "gx" + ps, gy = "gy" + ps;
-          o << ind << "  if (edge_tile) {\n";
-          o << ind << "  const bool wx = " << (p.bc[0] == KF_BC_PERIODIC ? "(" + gx + " < GX || " + gx + " >= NX - GX)" : "false")
-            << ", wy = " << (p.bc[1] == KF_BC_PERIODIC ? "(" + gy + " < GY || " + gy + " >= NY - GY)" : "false") << ";\n";
-          o << ind << "  if (wx || wy) {\n";
-          o << ind << "    const int gx2 = " << gx << " < GX ? " << gx << " + NX : " << gx << " - NX;\n";
-          o << ind << "    const int gy2 = " << gy << " < GY ? " << gy << " + NY : " << gy << " - NY;\n";
-          o << ind << "    const long long pb = (long long)pz" << uu << " * PLANE;\n";
-          for (auto& oi : outs)
-            if (oi.outi >= 0) {
-              o << ind << "    if (wx) a.out[" << oi.outi << "][pb + (long long)" << gy << " * PITCH + gx2] = " << vals[oi.stmt] << ";\n";
-              o << ind << "    if (wy) a.out[" << oi.outi << "][pb + (long long)gy2 * PITCH + " << gx << "] = " << vals[oi.stmt] << ";\n";
-              o << ind << "    if (wx && wy) a.out[" << oi.outi << "][pb + (long long)gy2 * PITCH + gx2] = " << vals[oi.stmt] << ";\n";
-            }
-          o << ind << "  }\n";
-          o << ind << "  }\n";
-        }
         o << ind << "}\n";
       }
     };
@@ -1424,6 +1356,40 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
       o << "   } }\n";
     }
     o << "  }\n";
+  }
+  // Periodic ghost copies of the live-outs (ghostwrite): after its whole z range, an edge tile copies
+  // the points it stored within the ghost width of a periodic x/y boundary to the opposite ghost
+  // layer (corners too), so the step needs no ghost-fill launches.  A separate epilogue keeps these
+  // scattered stores out of the compute loop's register budget; the values are re-read from global
+  // memory, written by this CTA before the barrier.
+  if (L.ghost_write && !L.live_out.empty()) {
+    const bool px_ = p.bc[0] == KF_BC_PERIODIC, py_ = p.bc[1] == KF_BC_PERIODIC;
+    o << "  if (edge_tile) {\n";
+    o << "    __syncthreads();\n";
+    o << "    const int tw = min(TX, NX - x0), th = min(TY, NY - y0), tzn = z1 - z0;\n";
+    // column strips (x) and row strips (y) of the tile inside the ghost width of a periodic boundary
+    o << "    const int xa0 = x0, xa1 = " << (px_ ? "min(GX, x0 + tw)" : "x0") << ";\n";
+    o << "    const int xb0 = " << (px_ ? "max(NX - GX, x0 + (xa1 > x0 ? xa1 - x0 : 0))" : "x0 + tw") << ", xb1 = x0 + tw;\n";
+    o << "    const int ya0 = y0, ya1 = " << (py_ ? "min(GY, y0 + th)" : "y0") << ";\n";
+    o << "    const int yb0 = " << (py_ ? "max(NY - GY, y0 + (ya1 > y0 ? ya1 - y0 : 0))" : "y0 + th") << ", yb1 = y0 + th;\n";
+    o << "    const int ncx = max(xa1 - xa0, 0) + max(xb1 - xb0, 0), ncy = max(ya1 - ya0, 0) + max(yb1 - yb0, 0);\n";
+    o << "    const int per = ncx * th + tw * ncy;\n";
+    o << "    for (int i = tid; i < per * tzn; i += NT) {\n";
+    o << "      const int zz = i / per, r = i - zz * per;\n";
+    o << "      int gx, gy;\n";
+    o << "      if (r < ncx * th) { const int c = r / th; gy = y0 + (r - c * th); gx = c < max(xa1 - xa0, 0) ? xa0 + c : xb0 + c - max(xa1 - xa0, 0); }\n";
+    o << "      else { const int q = r - ncx * th, c = q / tw; gx = x0 + (q - c * tw); gy = c < max(ya1 - ya0, 0) ? ya0 + c : yb0 + c - max(ya1 - ya0, 0); }\n";
+    o << "      const bool wx = " << (px_ ? "(gx < GX || gx >= NX - GX)" : "false") << ", wy = "
+      << (py_ ? "(gy < GY || gy >= NY - GY)" : "false") << ";\n";
+    o << "      const int gx2 = gx < GX ? gx + NX : gx - NX, gy2 = gy < GY ? gy + NY : gy - NY;\n";
+    o << "      const long long pb = (long long)(z0 + zz) * PLANE;\n";
+    for (size_t oi = 0; oi < L.live_out.size(); oi++) {
+      o << "      { const real v = a.out[" << oi << "][pb + (long long)gy * PITCH + gx];\n";
+      o << "        if (wx) a.out[" << oi << "][pb + (long long)gy * PITCH + gx2] = v;\n";
+      o << "        if (wy) a.out[" << oi << "][pb + (long long)gy2 * PITCH + gx] = v;\n";
+      o << "        if (wx && wy) a.out[" << oi << "][pb + (long long)gy2 * PITCH + gx2] = v; }\n";
+    }
+    o << "    }\n  }\n";
   }
   o << "}\n";
   cg.source = o.str();
