@@ -78,7 +78,25 @@ def _region(prog: Program, tile_lo, tile_hi, ext) -> Optional[List[np.ndarray]]:
     return ax
 
 
-def run_group_tiles(prog: Program, grp: List[int], mem: _Mem, params, tile, order) -> None:
+def refill_ghosts(prog: Program, mem: _Mem) -> None:
+    """Ghost-limited mode: before a group, every buffer's ghost layer on PERIODIC axes is refreshed
+    with the wrapped interior (what the device's ghost fills / ghost writes / halo exchanges
+    provide), one axis after the other (x, then y over whole padded rows, then z planes)."""
+    n, g = prog.n, prog.ghost
+    for b in mem.buf.values():
+        for a in range(3):
+            if prog.bc[a] != BC_PERIODIC or g[a] == 0:
+                continue
+            ax = 2 - a
+            lo = [slice(None)] * 3
+            src = [slice(None)] * 3
+            lo[ax], src[ax] = slice(0, g[a]), slice(n[a], n[a] + g[a])
+            b[tuple(lo)] = b[tuple(src)]
+            lo[ax], src[ax] = slice(g[a] + n[a], n[a] + 2 * g[a]), slice(g[a], 2 * g[a])
+            b[tuple(lo)] = b[tuple(src)]
+
+
+def run_group_tiles(prog: Program, grp: List[int], mem: _Mem, params, tile, order, ghost_limited=False) -> None:
     ext, _ = L.extended_regions(prog, grp)
     lout = L.live_out(prog, grp)
     n = prog.n
@@ -94,7 +112,19 @@ def run_group_tiles(prog: Program, grp: List[int], mem: _Mem, params, tile, orde
 
     def hbm_load(x, v, qx, qy, qz):
         b = mem.get(x, v)
-        return b[np.ix_(wrapped(2, qz) + g[2], wrapped(1, qy) + g[1], wrapped(0, qx) + g[0])]
+        if not ghost_limited:
+            return b[np.ix_(wrapped(2, qz) + g[2], wrapped(1, qy) + g[1], wrapped(0, qx) + g[0])]
+        # V6 pin: periodic neighbours only through the stored ghost layer of width ghost[a]; a read
+        # beyond it has no defined value (NaN sentinel)
+        idx, ok = [], []
+        for a, q in ((2, qz), (1, qy), (0, qx)):
+            i = q + g[a]
+            ok.append((i >= 0) & (i < n[a] + 2 * g[a]))
+            idx.append(np.clip(i, 0, n[a] + 2 * g[a] - 1))
+        val = b[np.ix_(*idx)].copy()
+        bad = ~(ok[0][:, None, None] & ok[1][None, :, None] & ok[2][None, None, :])
+        val[bad] = np.nan
+        return val
 
     def compute_tile(t):
         tlo = [t[a] * tile[a] for a in range(3)]
@@ -166,8 +196,10 @@ def n_tiles(prog: Program, tile) -> int:
 
 
 def run_fused(prog: Program, plan: List[int], inputs: Dict[str, np.ndarray], nsteps: int, tile,
-              order="snapshot", params=None) -> Dict[str, np.ndarray]:
-    """Run `nsteps` of the fused plan (groups in quotient-topological order, R18)."""
+              order="snapshot", params=None, ghost_limited=False) -> Dict[str, np.ndarray]:
+    """Run `nsteps` of the fused plan (groups in quotient-topological order, R18).  ghost_limited:
+    periodic reads go through ghost layers of the declared width, refreshed before every group
+    (the semantic pin of V6's ghost rule)."""
     params = list(prog.params if params is None else params)
     mem = _Mem(prog, inputs)
     gs = L.groups_of(plan)
@@ -176,6 +208,8 @@ def run_fused(prog: Program, plan: List[int], inputs: Dict[str, np.ndarray], nst
     with np.errstate(all="ignore"):
         for _ in range(nsteps):
             for g in qo:
-                run_group_tiles(prog, gs[g], mem, params, tile, order)
+                if ghost_limited:
+                    refill_ghosts(prog, mem)
+                run_group_tiles(prog, gs[g], mem, params, tile, order, ghost_limited)
             mem.end_step()
     return {nm: mem.buf[i] for i, (nm, _) in enumerate(prog.arrays)}

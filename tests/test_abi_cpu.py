@@ -231,7 +231,16 @@ def test_paper_projection_abi_matches_oracle_and_example():
     assert out.b_sh == 688 == ref["b_sh"]
     assert out.p_membound_gflops == ref["p_membound_gflops"]
     assert out.t_pro_s == ref["t_pro_s"]
-    assert out.eq2_ok and out.eq3_ok is not None
+    # Eq. 2/3/6/7 verdicts and T_pro against the hand calculation (tests/golden/eq10_hand_calc.json)
+    hand = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "eq10_hand_calc.json")))
+    for k, v in hand["inputs"].items():
+        setattr(m, k, v)
+    assert lib().kf_paper_projection(ctypes.byref(m), ctypes.byref(out)) == 0
+    e = hand["expected"]
+    assert (out.h_th, out.b_sh, out.b_eff, out.p_membound_gflops) == (e["h_th"], e["b_sh"], e["b_eff"], e["p_membound_gflops"])
+    assert out.t_pro_s == pytest.approx(e["t_pro_s"], rel=1e-15, abs=0)
+    assert (bool(out.eq2_ok), bool(out.eq3_ok), bool(out.eq6_ok), bool(out.eq7_ok)) == \
+        (e["eq2_ok"], e["eq3_ok"], e["eq6_ok"], e["eq7_ok"])
 
 
 def test_target_knobs_validated():

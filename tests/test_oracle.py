@@ -365,6 +365,40 @@ def test_tile_simulator_pins_V5(seed):
     assert checked >= 1
 
 
+def test_tile_simulator_pins_V6_ghost_rule():
+    """Semantic pin of V6 (O-7, ghost-limited mode): periodic neighbours are read only through the
+    stored ghost layer (width `ghost`, refreshed before every group as the device does).  For plans
+    passing V1-V5: V6 legal  <=>  the fused execution reproduces the unfused interpreter bit for
+    bit; a plan whose accumulated input halo exceeds the ghost width reads past the ghost layer."""
+    n_v6 = n_ok = 0
+    for seed in range(12):
+        rng = np.random.default_rng(500 + seed)
+        bc = (1, 1, int(rng.integers(0, 2)))
+        flags = [0, PROG_RELAX_EXPANDABLE, PROG_RELAX_ALL][seed % 3]
+        prog = P.random_program(900 + seed, nk=4, na=4, n=(6, 5, 4), bc=bc, flags=flags, max_r=1)
+        inp = D.uniform(prog, seed)
+        ref = interp.run(prog, inp, 2)
+        live = [nm for x, (nm, _) in enumerate(prog.arrays) if G.step_live(prog, x) or not G.writers(prog, x)]
+        for plan in En.restricted_growth(len(prog.kernels)):
+            v = L.validate(prog, plan)
+            if v[0] not in (L.V_OK, L.V6_HALO):
+                continue
+            out = TS.run_fused(prog, plan, inp, 2, (3, 2, 2), "snapshot", ghost_limited=True)
+            # periodic ghost layers hold refreshed wraps here (the device's too, R9): compare the
+            # interior and the frozen ghosts
+            m = np.ones(prog.padded_shape(), bool)
+            for a in range(3):
+                if prog.bc[a] == 1:
+                    sl = [slice(None)] * 3
+                    sl[2 - a] = np.r_[0:prog.ghost[a], prog.n[a] + prog.ghost[a]:prog.n[a] + 2 * prog.ghost[a]]
+                    m[tuple(sl)] = False
+            exact = all(np.array_equal(bits(out[nm][m]), bits(ref[nm][m])) for nm in live)
+            assert exact == (v[0] == L.V_OK), (seed, plan, v)
+            n_v6 += v[0] == L.V6_HALO
+            n_ok += v[0] == L.V_OK
+    assert n_v6 >= 5 and n_ok >= 20, (n_v6, n_ok)
+
+
 def test_tile_simulator_fig3_and_tiny():
     for prog, plan, nsteps in ((P.fig3(n=(8, 6, 4)), P.FIG3_PLAN_XY, 1), (P.tiny(n=(8, 8, 8)), [0, 0, 1], 3)):
         inp = D.inputs_for(prog, 3)
@@ -467,6 +501,25 @@ def test_paper_eq8_worked_example_golden():
     assert r["b_sh"] == gold["printed"]["b_sh"]
     assert r["p_membound_gflops"] == 688 * 14 * 202 / (8 * 128 * 64) == gold["derived_from_printed_formula"]["p_membound_gflops"]
     assert round(100 * r["p_membound_gflops"] / gold["printed"]["roofline_gflops"], 2) == gold["derived_from_printed_formula"]["percent"]
+
+
+def test_paper_eq10_hand_calculation_golden():
+    """NEXT-2 pin of T_pro (Eq. 10) under reading R12, against the hand calculation in
+    tests/golden/eq10_hand_calc.json (exact rational arithmetic written out step by step)."""
+    from oracle import paper_model
+    gold = json.load(open(os.path.join(GOLD, "eq10_hand_calc.json")))
+    i = gold["inputs"]
+    r = paper_model.project(**{k: i[k] for k in ("t_b", "blocks_smx", "thr", "blocks", "hal", "halo", "shared_arrays",
+                                                 "smx", "gmem_bw_gbs", "elem_bytes", "fl_unfused_sum", "flop_halo_sum")})
+    e = gold["expected"]
+    assert r["h_th"] == e["h_th"] and r["b_sh"] == e["b_sh"] and r["b_eff"] == e["b_eff"]
+    assert r["p_membound_gflops"] == e["p_membound_gflops"]
+    assert r["t_pro_s"] == pytest.approx(e["t_pro_s"], rel=1e-15, abs=0)
+    # no halo layer (c = 0): T_pro is the unfused FLOPs over P_MemBound with B_Sh = T_B*Blocks/|ShrLst|
+    r0 = paper_model.project(**dict({k: i[k] for k in ("t_b", "blocks_smx", "thr", "blocks", "hal", "shared_arrays",
+                                                       "smx", "gmem_bw_gbs", "elem_bytes", "fl_unfused_sum",
+                                                       "flop_halo_sum")}, halo=0))
+    assert r0["b_sh"] == 86 * 32 / 2 and r0["t_pro_s"] < r["t_pro_s"]
 
 
 def test_suite_generator_thread_load_and_sharing_sets():
