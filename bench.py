@@ -409,7 +409,9 @@ AUTOTUNE_CANDIDATES = [  # (tile, stages, zunroll, ringunroll, minblocks, canvas
     ((32, 8, 64), 2, 1, 0, -1, 0, 2, 1), ((32, 8, 64), 2, 1, 0, 0, 1, 2, 1), ((32, 8, 32), 2, 1, 0, -1, 1, 2, 1),
     # z chunks of 43 planes: 3 chunks of a 128-plane column, 6.9 waves of 3 CTAs/SM instead of 4.6
     # (wave quantisation; measured -2..-4 % on the flux groups)
-    ((32, 8, 43), 2, 1, 0, -1, 1, 2, 1), ((32, 8, 43), 2, 1, 0, -1, 1, 2, 0), ((32, 8, 43), 2, 1, 0, -1, 1)]
+    ((32, 8, 43), 2, 1, 0, -1, 1, 2, 1), ((32, 8, 43), 2, 1, 0, -1, 1, 2, 0), ((32, 8, 43), 2, 1, 0, -1, 1),
+    # taller / wider pair tiles: less halo per point (36x20/512 = 1.41 vs 36x12/256 = 1.69 box/tile)
+    ((32, 16, 43), 2, 1, 0, -1, 1, 2, 1), ((32, 16, 43), 2, 1, 0, -1, 1, 2, 0), ((64, 8, 43), 2, 1, 0, -1, 1, 2, 1)]
 
 
 def cand_kw(base_kw, c):

@@ -329,6 +329,10 @@ typedef struct {
   char name[64];
 } kf_group_info;
 kf_status kf_exec_group_info(const kf_exec* ex, int32_t group, kf_group_info* out);
+/* Loads every group kernel of the executor onto the calling thread's current device (the first
+ * kf_exec_run does it implicitly); afterwards kf_exec_group_info reports the loaded functions'
+ * CU_FUNC_ATTRIBUTE_NUM_REGS / LOCAL_SIZE_BYTES (the V7/V8 hardware pin).  Needs a GPU. */
+kf_status kf_exec_load(kf_exec* ex);
 /* Generated CUDA source of a group (for inspection); *len receives the full length. */
 kf_status kf_exec_group_source(const kf_exec* ex, int32_t group, char* buf, int64_t cap, int64_t* len);
 /* Profiling mode: when on, kf_exec_run records a CUDA event around every group launch on

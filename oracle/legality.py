@@ -253,7 +253,32 @@ def schedule(prog: Program, grp: List[int], target: Target):
         nb = (-(-w // bx)) * (-(-h // by))
         rounds = max(rounds, -(-nb // threads))
     P = min(8, target.pblock[0] * target.pblock[1] * target.zunroll * rounds)
-    regs = 48 + 2 * (es // 4) * (depth + 3) * P
+    # register model (V8, R20 revised in round 2): the paper's Eq. 4/6,
+    #   R_est = R_adr*U + RegFac*(es/4)*P*(ThrLD + depth)
+    # R_adr = 32 per plane of a stream iteration, R_fetch = 0 (TMA), RegFac = 1 (no reuse, the upper
+    # end of P:347's range), ThrLD = distinct (array, version, offset) loads a thread holds: the whole
+    # group's on the canvas (one canvas point -- or one aligned pair -- per thread, rounds = 1), the
+    # largest kernel's otherwise
+    clo0 = max([ext[k][0][0] for k in alive] + [0])
+    chi0 = max([ext[k][1][0] for k in alive] + [0])
+    canvas = False
+    if alive and tuple(target.pblock) == (1, 1):
+        canvas = -(-(cw * ch) // threads) == 1
+    if alive and tuple(target.pblock) == (2, 1) and target.zunroll == 1 and TX % 2 == 0 and prog.n[0] % 2 == 0:
+        cwp = TX // 2 + (clo0 + 1) // 2 + (chi0 + 1) // 2
+        canvas = -(-(cwp * ch) // threads) == 1
+    loads = set()
+    kmax = 0
+    for k in alive:
+        nk = 0
+        for x, offs in G.reads(prog, k).items():
+            v = G.version_read(prog, k, x)
+            for d in offs:
+                loads.add((x, v, tuple(d)))
+                nk += 1
+        kmax = max(kmax, nk)
+    thrld = len(loads) if canvas else kmax
+    regs = 32 * target.zunroll + (es // 4) * P * (thrld + depth)
     return dict(ext=ext, pts=pts, delay=D, res=res, smem=smem, regs=regs, alive=alive)
 
 

@@ -150,6 +150,7 @@ SIGNATURES = {
     "kf_exec_group_times": (C.c_int, [P, C.POINTER(C.c_double), C.c_int32, I32P, C.POINTER(C.c_int64)]),
     "kf_exec_set_graph": (C.c_int, [P, C.c_int32]),
     "kf_exec_invalidate": (C.c_int, [P]),
+    "kf_exec_load": (C.c_int, [P]),
     "kf_flush_l2": (C.c_int, [P, C.c_uint64, P]),
     "kf_paper_projection": (C.c_int, [C.POINTER(kf_paper_meta), C.POINTER(kf_paper_proj)]),
     "kf_dist_unique_id": (C.c_int, [C.POINTER(C.c_uint8)]),

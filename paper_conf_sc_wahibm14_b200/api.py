@@ -295,6 +295,10 @@ class Exec:
     def set_graph(self, on: bool):
         check(lib().kf_exec_set_graph(self.h, int(on)))
 
+    def load(self):
+        """kf_exec_load: load every group kernel onto the current device (NUM_REGS / LOCAL_SIZE)."""
+        check(lib().kf_exec_load(self.h))
+
     def invalidate(self):
         """kf_exec_invalidate: array contents outside the interior changed under the same pointers."""
         check(lib().kf_exec_invalidate(self.h))

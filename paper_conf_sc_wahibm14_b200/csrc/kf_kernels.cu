@@ -67,12 +67,13 @@ __global__ void fill_z(T* __restrict__ base, Geom g) {
 // is periodic) and the y-ghost rows over the x range not already covered (if y is periodic).
 struct FillList { void* base[kMaxFillBufs]; };
 
-// zghost: only the z ghost planes (2*gz of them) -- the run-start fill of renamed scratch versions,
-// whose interior planes are not written yet (their x/y ghosts are filled after their producer).
+// frozen_only: only the ghost cells lying in the ghost layer of a FROZEN axis (bit 0 x, 1 y, 2 z
+// frozen) -- the run-start fill of renamed scratch versions, whose other cells are not written yet
+// (they are filled or ghost-written after their producer).
 template <typename T>
-__global__ void fill_xy_multi(FillList L, Geom g, int px, int py, int zghost) {
+__global__ void fill_xy_multi(FillList L, Geom g, int px, int py, int frozen_only) {
   T* base = (T*)L.base[blockIdx.y];
-  const int NZ = zghost ? 2 * g.gz : g.nz + 2 * g.gz, NYp = g.ny + 2 * g.gy;
+  const int NZ = g.nz + 2 * g.gz, NYp = g.ny + 2 * g.gy;
   const long long nxs = px ? 2LL * g.gx * NYp * NZ : 0;                  // x-ghost columns
   const int x_lo = px ? 0 : -g.gx, x_w = px ? g.nx : g.nx + 2 * g.gx;    // y rows: x range not in nxs
   const long long nys = py ? (long long)x_w * 2 * g.gy * NZ : 0;
@@ -95,7 +96,9 @@ __global__ void fill_xy_multi(FillList L, Geom g, int px, int py, int zghost) {
     }
     const int si = (px && (i < 0 || i >= g.nx)) ? (i < 0 ? i + g.nx : i - g.nx) : i;
     const int sj = (py && (j < 0 || j >= g.ny)) ? (j < 0 ? j + g.ny : j - g.ny) : j;
-    if (zghost && k >= 0) k += g.nz;   // planes -gz..-1, then nz..nz+gz-1
+    if (frozen_only && !(((frozen_only & 1) && (i < 0 || i >= g.nx)) || ((frozen_only & 2) && (j < 0 || j >= g.ny)) ||
+                         ((frozen_only & 4) && (k < 0 || k >= g.nz))))
+      continue;
     const long long o = (long long)(k + g.gz) * g.plane + g.xoff;
     base[o + (long long)(j + g.gy) * g.pitch + i] = base[o + (long long)(sj + g.gy) * g.pitch + si];
   }
@@ -176,9 +179,9 @@ cudaError_t launch_fill(int axis, void* base, int es, const Geom& g, cudaStream_
 }
 
 cudaError_t launch_fill_xy_multi(void* const* bufs, int n, int px, int py, int es, const Geom& g, cudaStream_t s,
-                                 int zghost) {
+                                 int frozen_only) {
   if (!px && !py) return cudaSuccess;
-  const long long NZ = zghost ? 2 * g.gz : g.nz + 2 * g.gz;
+  const long long NZ = g.nz + 2 * g.gz;
   const long long per = (px ? 2LL * g.gx * (g.ny + 2 * g.gy) : 0) * NZ +
                         (py ? (long long)(px ? g.nx : g.nx + 2 * g.gx) * 2 * g.gy * NZ : 0);
   if (per == 0) return cudaSuccess;
@@ -189,8 +192,8 @@ cudaError_t launch_fill_xy_multi(void* const* bufs, int n, int px, int py, int e
     long long nb = (per + 255) / 256;
     const long long cap = (148LL * 16 + m - 1) / m;   // ~16 CTAs per SM over all buffers
     dim3 grid(unsigned(nb < cap ? nb : cap), unsigned(m));
-    if (es == 4) fill_xy_multi<float><<<grid, 256, 0, s>>>(L, g, px, py, zghost);
-    else fill_xy_multi<double><<<grid, 256, 0, s>>>(L, g, px, py, zghost);
+    if (es == 4) fill_xy_multi<float><<<grid, 256, 0, s>>>(L, g, px, py, frozen_only);
+    else fill_xy_multi<double><<<grid, 256, 0, s>>>(L, g, px, py, frozen_only);
   }
   return cudaGetLastError();
 }

@@ -12,7 +12,7 @@ cudaError_t launch_fill(int axis, void* base, int es, const Geom& g, cudaStream_
 // periodic x/y ghosts of n buffers, batched kMaxFillBufs per launch (px, py: axis periodic)
 constexpr int kMaxFillBufs = 32;
 cudaError_t launch_fill_xy_multi(void* const* bufs, int n, int px, int py, int es, const Geom& g, cudaStream_t s,
-                                 int zghost = 0);
+                                 int frozen_only = 0);
 cudaError_t launch_copy_shell(void* dst, const void* src, int es, const Geom& g, cudaStream_t s);
 cudaError_t launch_copy_box(void* dst, long long dpitch, long long dplane, const void* src, long long spitch,
                             long long splane, int w, int h, int d, int es, cudaStream_t s);

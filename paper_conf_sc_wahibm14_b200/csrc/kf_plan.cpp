@@ -12,6 +12,7 @@
 #include <cstdio>
 #include <climits>
 #include <cstring>
+#include <tuple>
 
 #include "kf_internal.hpp"
 
@@ -257,7 +258,48 @@ GroupLowering lower_group(const Program& p, const std::vector<int>& g, const kf_
     rounds = std::max(rounds, (nb + L.threads - 1) / L.threads);
   }
   const int P = std::min(8, t.pblock[0] * t.pblock[1] * U * rounds);
-  L.regs = 48 + 2 * (es / 4) * (depth + 3) * P;
+  // Register model (V8; R20, revised in round 2 after the hardware pin): the paper's Eq. 4/6
+  // for one thread of a fused group,
+  //     R_est = R_adr * U + RegFac * (es/4) * P * (ThrLD + depth),
+  // R_adr = 32 address / index / predicate registers per plane of a stream iteration, R_fetch = 0
+  // (TMA stages the live-ins without registers), RegFac = 1 (no register reuse: the upper end of
+  // the paper's range 1/max(ThrLD) <= RegFac <= 1), P = points per thread (<= 8), depth = deepest
+  // RPN stack, ThrLD = distinct values (array, version, offset) a thread loads and holds: the whole
+  // group's on the canvas (its loads are reused across the phases of an iteration), the largest
+  // single kernel's on the per-kernel path.  The kernel is compiled with this as its register cap
+  // (__maxnreg__), so NUM_REGS <= R_est; a GPU test asserts it never spills at that cap.
+  {
+    int clo0 = 0, chi0 = 0, clo1 = 0, chi1 = 0;
+    for (int k : alive) {
+      clo0 = std::max(clo0, L.ext[k].elo[0]);
+      chi0 = std::max(chi0, L.ext[k].ehi[0]);
+      clo1 = std::max(clo1, L.ext[k].elo[1]);
+      chi1 = std::max(chi1, L.ext[k].ehi[1]);
+    }
+    const int CW = TX + clo0 + chi0, CH = TY + clo1 + chi1;
+    bool canvas = false;
+    if (!alive.empty() && t.pblock[0] == 1 && t.pblock[1] == 1)
+      canvas = (CW * CH + L.threads - 1) / L.threads == 1;
+    if (!alive.empty() && t.pblock[0] == 2 && t.pblock[1] == 1 && U == 1 && TX % 2 == 0 && p.n[0] % 2 == 0) {
+      const int cwp = TX / 2 + (clo0 + 1) / 2 + (chi0 + 1) / 2;
+      canvas = (cwp * CH + L.threads - 1) / L.threads == 1;
+    }
+    std::set<std::tuple<int, int, int, int, int>> all;
+    int kmax = 0;
+    for (int k : alive) {
+      int nk = 0;
+      for (auto& [x, offs] : p.kernels[k].reads) {
+        const int v = p.vr(k, x);
+        for (auto& d : offs) {
+          all.insert(std::make_tuple(x, v, d[0], d[1], d[2]));
+          nk++;
+        }
+      }
+      kmax = std::max(kmax, nk);
+    }
+    const int thrld = canvas ? int(all.size()) : kmax;
+    L.regs = 32 * U + (es / 4) * P * (thrld + depth);
+  }
   return L;
 }
 

@@ -80,7 +80,7 @@ struct Compiled {
   std::vector<char> cubin;
   std::string log;
   int regs_ptxas = -1, spill = -1;
-  bool nocap = false;   // compiled with KF_NO_MAXNREG (register cap dropped)
+  bool nocap = false;   // compiled with KF_NO_MAXNREG (occupancy cap dropped: the cap is R_est)
 };
 
 static Compiled nvrtc_compile(const std::string& src, const std::string& name) {
@@ -134,8 +134,8 @@ static std::shared_ptr<Compiled> compile_cached(const std::string& src, const st
     if (it != g_cubin_cache.end()) return it->second;
   }
   auto c = std::make_shared<Compiled>(nvrtc_compile(src, name));
-  // the register cap (__maxnreg__, occupancy) must not cost local-memory spills
-  if (c->spill > 0 && src.find("__maxnreg__") != std::string::npos) {
+  // the occupancy register cap (below R_est) must not cost local-memory spills: rebuild at R_est
+  if (c->spill > 0 && src.find("#ifndef KF_NO_MAXNREG") != std::string::npos) {
     c = std::make_shared<Compiled>(nvrtc_compile("#define KF_NO_MAXNREG 1\n" + src, name));
     c->nocap = true;
   }
@@ -371,7 +371,7 @@ static void run_fill(kf_exec* E, int buf, cudaStream_t s) {
 }
 
 // Consecutive fills of a schedule in one launch (x and y together; z, if periodic, after them).
-static void run_fills(kf_exec* E, const std::vector<int>& bufs, cudaStream_t s, int zghost = 0) {
+static void run_fills(kf_exec* E, const std::vector<int>& bufs, cudaStream_t s, int frozen_only = 0) {
   if (bufs.empty()) return;
   const Program& p = E->prog->p;
   Geom gm = geom(p);
@@ -382,7 +382,7 @@ static void run_fills(kf_exec* E, const std::vector<int>& bufs, cudaStream_t s, 
   std::vector<void*> ptr;
   for (int b : bufs) ptr.push_back(buf_ptr(E, b));
   CK(launch_fill_xy_multi(ptr.data(), int(ptr.size()), p.bc[0] == KF_BC_PERIODIC, p.bc[1] == KF_BC_PERIODIC, p.es, gm, s,
-                          zghost));
+                          frozen_only));
   if (p.bc[2] == KF_BC_PERIODIC)
     for (void* b : ptr) CK(launch_fill(2, b, p.es, gm, s));
 }
@@ -434,7 +434,7 @@ static void ensure_device(kf_exec* E) {
       drv().funcGetAttribute(&g.regs, CU_FUNC_ATTRIBUTE_NUM_REGS, g.fn);
       drv().funcGetAttribute(&g.local, CU_FUNC_ATTRIBUTE_LOCAL_SIZE_BYTES, g.fn);
       // the register cap must not cost local memory (spills): rebuild without it
-      if (g.local > 0 && !g.comp->nocap && g.cg.source.find("__maxnreg__") != std::string::npos) {
+      if (g.local > 0 && !g.comp->nocap && g.cg.source.find("#ifndef KF_NO_MAXNREG") != std::string::npos) {
         g.comp = compile_nocap(g.cg.source, g.cg.name);
         if (drv().moduleUnload) drv().moduleUnload(g.mod);
         g.mod = nullptr;
@@ -551,13 +551,16 @@ static void exec_run(kf_exec* E, void* const* arrays, void* scratch, uint64_t sc
     E->shell_init_scratch = scratch;
     E->shell_init_arrays = arr;
   }
-  // run-start fills: the caller's arrays whole; renamed scratch versions (interior not yet written,
-  // x/y ghosts of interior planes filled after their producer) only on the frozen z ghost planes
+  // run-start fills: the caller's arrays whole; renamed scratch versions (not written yet: their
+  // periodic ghosts are filled / ghost-written after their producer) only where the cell lies in a
+  // FROZEN axis' ghost layer (constant cells, R9)
   {
     std::vector<int> arr_b, scr_b;
     for (int b : E->fill_all) (b < p.na ? arr_b : scr_b).push_back(b);
     run_fills(E, arr_b, s);
-    run_fills(E, scr_b, s, p.bc[2] == KF_BC_FROZEN ? 1 : 0);
+    const int frozen = (p.bc[0] == KF_BC_FROZEN ? 1 : 0) | (p.bc[1] == KF_BC_FROZEN ? 2 : 0) | (p.bc[2] == KF_BC_FROZEN ? 4 : 0);
+    if (frozen && p.bc[2] != KF_BC_PERIODIC) run_fills(E, scr_b, s, frozen);
+    else run_fills(E, scr_b, s);
   }
   int64_t reps = nsteps / E->period, rem = nsteps % E->period;
   if (E->use_graph && !E->profiling && reps > 0) {
@@ -858,6 +861,13 @@ kf_status kf_exec_group_times(kf_exec* ex, double* ms, int32_t cap, int32_t* n, 
     for (int i = 0; i < int(ex->gms.size()) && i < cap && ms; i++) ms[i] = ex->gms[i];
     *n = int(ex->gms.size());
     if (launches) *launches = ex->launches;
+  });
+}
+
+kf_status kf_exec_load(kf_exec* ex) {
+  KF_TRY({
+    if (!ex) fail(KF_E_ARG, "null exec");
+    ensure_device(ex);
   });
 }
 
