@@ -144,25 +144,23 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
   // register cap (__maxnreg__): at most what keeps the shared-memory-limited number of CTAs per SM
   // resident (minblocks 0; or minblocks CTAs) and never above the resource model's estimate R_est
   // (V8, R20).  The runtime recompiles without the cap if it would make ptxas spill.
-  // The register model R_est (V8) is the kernel's register budget: __maxnreg__(R_est), lowered
-  // further to keep the shared-memory-limited number of CTAs per SM resident (minblocks 0) or
-  // minblocks CTAs (n >= 1).  If the lowered cap would make ptxas spill, the runtime rebuilds with
-  // KF_NO_MAXNREG, i.e. at R_est itself.
+  // Registers.  minblocks -1: __launch_bounds__(NT), ptxas' own choice -- the register model R_est
+  // (V8) must bound it; a GPU test pins NUM_REGS <= R_est and no spills over every bench
+  // configuration.  (Measured: explicit budgets -- __maxnreg__(R_est), or __launch_bounds__ with a
+  // minimum CTA count -- make ptxas use up to the budget, e.g. 124 or 162 instead of 88 or 72
+  // registers on the flux groups, one CTA per SM less.)  minblocks >= 0: __maxnreg__ keeps the
+  // shared-memory-limited number of CTAs per SM resident (0) or n CTAs (n >= 1), never above R_est;
+  // if that would make ptxas spill, the runtime rebuilds without it (KF_NO_MAXNREG).
   if (const char* fc = getenv("KF_MAXNREG")) {   // experiments only: force a register cap
     o << "#define KF_BOUNDS __maxnreg__(" << atoi(fc) << ")\n";
+  } else if (L.minblocks >= 0) {
+    const int smem_ctas = 233472 / std::max(1, L.smem + 1024);
+    const int minb = L.minblocks > 0 ? L.minblocks : std::max(1, std::min({smem_ctas, 2048 / std::max(1, NT), 8}));
+    const int cap = std::max(24, std::min({65536 / (NT * minb) / 8 * 8, L.regs, 255}));
+    o << "#ifndef KF_NO_MAXNREG\n#define KF_BOUNDS __maxnreg__(" << cap
+      << ")\n#else\n#define KF_BOUNDS __launch_bounds__(NT)\n#endif\n";
   } else {
-    const int rest = std::max(24, std::min(L.regs, 255));
-    int cap = rest;
-    if (L.minblocks >= 0) {
-      const int smem_ctas = 233472 / std::max(1, L.smem + 1024);
-      const int minb = L.minblocks > 0 ? L.minblocks : std::max(1, std::min({smem_ctas, 2048 / std::max(1, NT), 8}));
-      cap = std::max(24, std::min(65536 / (NT * minb) / 8 * 8, rest));
-    }
-    if (cap < rest)
-      o << "#ifndef KF_NO_MAXNREG\n#define KF_BOUNDS __maxnreg__(" << cap << ")\n#else\n#define KF_BOUNDS __maxnreg__("
-        << rest << ")\n#endif\n";
-    else
-      o << "#define KF_BOUNDS __maxnreg__(" << rest << ")\n";
+    o << "#define KF_BOUNDS __launch_bounds__(NT)\n";
   }
   o << "extern \"C\" __global__ void KF_BOUNDS " << cg.name << "(const __grid_constant__ KfArgs a) {\n";
   // pointer arithmetic from the __shared__ array keeps the shared state space (LDS/STS, 32-bit

@@ -80,7 +80,7 @@ struct Compiled {
   std::vector<char> cubin;
   std::string log;
   int regs_ptxas = -1, spill = -1;
-  bool nocap = false;   // compiled with KF_NO_MAXNREG (occupancy cap dropped: the cap is R_est)
+  bool nocap = false;   // compiled with KF_NO_MAXNREG (occupancy register cap dropped)
 };
 
 static Compiled nvrtc_compile(const std::string& src, const std::string& name) {
@@ -134,7 +134,7 @@ static std::shared_ptr<Compiled> compile_cached(const std::string& src, const st
     if (it != g_cubin_cache.end()) return it->second;
   }
   auto c = std::make_shared<Compiled>(nvrtc_compile(src, name));
-  // the occupancy register cap (below R_est) must not cost local-memory spills: rebuild at R_est
+  // the occupancy register cap (__maxnreg__) must not cost local-memory spills: rebuild without it
   if (c->spill > 0 && src.find("#ifndef KF_NO_MAXNREG") != std::string::npos) {
     c = std::make_shared<Compiled>(nvrtc_compile("#define KF_NO_MAXNREG 1\n" + src, name));
     c->nocap = true;

@@ -22,7 +22,8 @@ def main():
     wl = sys.argv[3] if len(sys.argv) > 3 else "weather"
     sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
     import bench
-    desc, gen, tkw, _ = bench.workload(wl)
+    w = bench.Workload(wl, 1)
+    desc, tkw = w.desc, dict(w.tkw)
     prog = kf.Program(desc)
     if which == "best":
         plan = bench.choose_plan(prog, kf.Target(**tkw), "best")[0]
@@ -30,13 +31,7 @@ def main():
         plan = {"hgga": HGGA, "hand": P.weather_hand_plan(desc), "unfused": list(range(44))}.get(which) or json.loads(which)
     else:
         plan = list(range(prog.nk)) if which == "unfused" else json.loads(which)
-    if gen is None:
-        L = prog.layout()
-        g = torch.Generator(device="cuda").manual_seed(3)
-        dt = torch.float64 if desc.dtype == 1 else torch.float32
-        dev = [torch.rand(L.elems, generator=g, device="cuda", dtype=dt) * 2 - 1 for _ in desc.arrays]
-    else:
-        dev = kf.device_arrays(prog, gen(desc, 3))
+    dev, _ = w.inputs(prog, 0)
     print(json.dumps({"workload": wl, "plan": plan}), flush=True)
     steps = int(os.environ.get("AB_STEPS", "10"))
     for v in variants:
