@@ -506,7 +506,10 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
                         const Ring& RR = L.rings[key.ring];
                         const long long amin = (long long)key.off * p.es;
                         const long long amax = ((long long)(CH - 1) * RR.px + (cv.cw - 1) + key.off + 1) * p.es;
-                        const bool nopred = L.canvas_ld && amin >= 0 && amax <= RR.plane_bytes;
+                        const bool anyring = getenv("KF_LD_ANYRING") != nullptr;   // A/B only: the racy round-1 rule
+                        const bool nopred = L.canvas_ld && (anyring ? RR.smem_off + amin >= 0 &&
+                                                                          RR.smem_off + (long long)(RR.slots - 1) * RR.plane_bytes + amax <= L.mbar_off
+                                                                    : amin >= 0 && amax <= RR.plane_bytes);
                         std::string ld = nopred ? acc
                                                 : "(ca" + rs + " && cx" + rs + " >= " + std::to_string(rc[0]) + " && cx" + rs + " < " +
                                                       std::to_string(rc[1]) + " && cy" + rs + " >= " + std::to_string(rc[2]) + " && cy" +
@@ -615,6 +618,8 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
     // inside the slot being read (see the single-point canvas above)
     const long long amin = (cxmin + rel) * p.es;
     const long long amax = ((long long)(CH - 1) * RR.px + cxmax + rel + 2) * p.es;
+    if (getenv("KF_LD_ANYRING"))   // A/B only: the racy round-1 rule
+      return L.canvas_ld && RR.smem_off + amin >= 0 && RR.smem_off + (long long)(RR.slots - 1) * RR.plane_bytes + amax <= L.mbar_off;
     return L.canvas_ld && amin >= 0 && amax <= RR.plane_bytes;
   };
   // z register queues of the pair canvas: a pair value (ring, po, rel) read at iteration t is the

@@ -86,10 +86,17 @@ def test_random_programs_random_legal_plans(seed):
     pb = [(1, 1), (2, 1), (2, 2), (1, 3)][seed % 4]
     ru = seed % 2
     gw = (seed // 2) % 2
+    ran = 0
     for plan in pick:
-        got, _ = run_kf(desc, plan, inputs, nsteps, kf.Target(tile=tile, zunroll=zu, pblock=pb, threads=64, ringunroll=ru,
-                                                              ghostwrite=gw))
+        t = kf.Target(tile=tile, zunroll=zu, pblock=pb, threads=64, ringunroll=ru, ghostwrite=gw)
+        if kf.Program(desc).validate(plan, t)[0] in (7, 8):   # resource model rejects this launch config
+            with pytest.raises(kf.KfError, match="KF_E_ILLEGAL_PLAN"):
+                kf.Exec(kf.Program(desc), plan, t)
+            t = kf.Target(tile=tile, zunroll=1, pblock=(1, 1), ringunroll=ru, ghostwrite=gw)
+        got, _ = run_kf(desc, plan, inputs, nsteps, t)
         assert compare(desc, got, ref) == [], (plan, tile)
+        ran += 1
+    assert ran >= 1
 
 
 def test_weather_small_fp64_plans():
@@ -263,7 +270,9 @@ def test_canvas_weather_knobs(cq, monkeypatch):
     ref = interp.run(desc, inputs, 2)
     prog = kf.Program(desc)
     tgt = kf.Target(tile=(32, 8, 0))
-    plans = [prog.search(kf.SEARCH_HGGA, tgt, seed=s)[0] for s in (1, 2)]
+    # plans searched for single points and for pairs (V8 differs: the pair canvas holds more values)
+    plans = [prog.search(kf.SEARCH_HGGA, tgt, seed=s)[0] for s in (1, 2)] + \
+        [prog.search(kf.SEARCH_HGGA, kf.Target(tile=(32, 8, 0), pblock=(2, 1)), seed=s)[0] for s in (1, 2)]
     for plan in plans:
         for kw in (dict(), dict(canvas_ld=0), dict(pblock=(2, 1)), dict(pblock=(2, 1), canvas_ld=0),
                    dict(pblock=(2, 1), pair_zq=0), dict(skew=1),

@@ -88,9 +88,9 @@ def test_ghostwrite_pair_canvas_drops_fills(ghost):
     inputs = D.inputs_for(desc, 21)
     ref = interp.run(desc, inputs, 3)
     prog = kf.Program(desc)
-    plan, _ = prog.search(kf.SEARCH_HGGA, kf.Target(tile=(32, 8, 0)), seed=2)
     for pb, zq in (((2, 1), 1), ((2, 1), 0), ((1, 1), 1)):
         tgt = kf.Target(tile=(32, 8, 0), pblock=pb, pair_zq=zq, ghostwrite=1, minblocks=-1)
+        plan, _ = prog.search(kf.SEARCH_HGGA, tgt, seed=2)      # legal under this launch config (V8)
         got, ex = run_kf(desc, plan, inputs, 3, tgt)
         assert ex.info().fills_per_step == 0
         from .gpu_util import compare
