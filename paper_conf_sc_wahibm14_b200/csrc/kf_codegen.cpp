@@ -218,6 +218,32 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
   for (auto& r : L.rings) canvas_pitches.insert(r.px);
   const bool pair_mode = canvas_mode && cv.pair;
   const int PSH = 2 * cv.lop - clo[0];   // pair mode: canvas x of the thread's first point = 2 * pair column - PSH
+  // Clamped canvas loads (canvas_ld): a lane outside the reading kernels' regions never stores (nor
+  // forwards to a stored point) what it computes, so it may load any address -- it loads the one of
+  // the nearest canvas point inside the regions' bounding rectangle (row and column clamped once,
+  // before the stream loop).  No predicate, no zeroing move, and every address stays inside the
+  // ring box of the plane being read, which no thread writes in the reading phase (an unclamped
+  // load on such a lane could reach a neighbouring ring that another kernel stores to: a race,
+  // compute-sanitizer racecheck, round 2).
+  std::map<std::array<int, 5>, std::string> clamp_base;   // {x0, x1, y0, y1, pitch} -> variable
+  std::string clamp_defs;
+  auto cbase = [&](const Rect& rc, int pitch) {
+    const std::array<int, 5> key{rc[0], rc[1], rc[2], rc[3], pitch};
+    auto it = clamp_base.find(key);
+    if (it != clamp_base.end()) return it->second;
+    const std::string nm = "ckb" + std::to_string(clamp_base.size());
+    const std::string cy = "min(max(cy_r0, " + std::to_string(rc[2]) + "), " + std::to_string(rc[3] - 1) + ")";
+    std::string cx;
+    if (pair_mode) {   // first-point x of an aligned pair inside [x0, x1): pair columns [lo, hi]
+      const int lo = (rc[0] + PSH + 1) >> 1, hi = (rc[1] - 1 + PSH) >> 1;
+      cx = "(2 * min(max(cxp_r0, " + std::to_string(lo) + "), " + std::to_string(std::max(lo, hi)) + ") - " + std::to_string(PSH) + ")";
+    } else {
+      cx = "min(max(cx_r0, " + std::to_string(rc[0]) + "), " + std::to_string(rc[1] - 1) + ")";
+    }
+    clamp_defs += "  const int " + nm + " = " + cy + " * " + std::to_string(pitch) + " + " + cx + ";\n";
+    clamp_base.emplace(key, nm);
+    return nm;
+  };
   if (pair_mode) {
     // pair mode: row-aligned threads over the tile's TX/2 pair columns, then the halo pair columns
     // (column-major); cx = canvas x of the first point (even tile-relative x: pairs are 16-byte
@@ -272,6 +298,7 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
           << " && cy" << rs << " >= " << oy << " && cy" << rs << " < " << oy + WY << ";\n";
       }
     }
+  o << "/*@@KF_CLAMP_BASES@@*/";
   o << "  __syncthreads();\n";
   // per-kernel compute / ghost plane ranges for this unit
   for (int k : alive) {
@@ -493,27 +520,16 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
                         std::string nm = key_name("cl", key, rs) + "_h" + std::to_string(ph);
                         const std::string acc = "P" + std::to_string(key.ring) + "_" + std::to_string(slot(key.ring, key.po)) +
                                                 "[cb" + std::to_string(L.rings[key.ring].px) + rs + " + " + std::to_string(key.off) + "]";
-                        // canvas_ld: a point outside the reading kernels' regions never stores (nor
-                        // forwards to a stored point) what it computes, so the load needs no predicate
-                        // if every address it can form, over all canvas points and ring slots, lies in
-                        // the rings' shared memory.  Saves the predicate and the zeroing move (ncu: 6 %
-                        // CS2R; g0 -14 %) but loads on lanes outside the regions: more wavefronts and
-                        // bank conflicts on the halo warp (+25 % shared wavefronts), so it is a per-group
-                        // launch knob chosen by measurement.
-                        // Every address must lie inside the slot being read (not merely inside the
-                        // rings): a slot is never written in the phase that reads it, while a
-                        // neighbouring ring or slot may be (compute-sanitizer racecheck, round 2).
+                        // canvas_ld: clamped unpredicated load (see cbase); else predicated with a zero
                         const Ring& RR = L.rings[key.ring];
-                        const long long amin = (long long)key.off * p.es;
-                        const long long amax = ((long long)(CH - 1) * RR.px + (cv.cw - 1) + key.off + 1) * p.es;
-                        const bool anyring = getenv("KF_LD_ANYRING") != nullptr;   // A/B only: the racy round-1 rule
-                        const bool nopred = L.canvas_ld && (anyring ? RR.smem_off + amin >= 0 &&
-                                                                          RR.smem_off + (long long)(RR.slots - 1) * RR.plane_bytes + amax <= L.mbar_off
-                                                                    : amin >= 0 && amax <= RR.plane_bytes);
-                        std::string ld = nopred ? acc
-                                                : "(ca" + rs + " && cx" + rs + " >= " + std::to_string(rc[0]) + " && cx" + rs + " < " +
-                                                      std::to_string(rc[1]) + " && cy" + rs + " >= " + std::to_string(rc[2]) + " && cy" +
-                                                      rs + " < " + std::to_string(rc[3]) + ") ? " + acc + " : (real)0";
+                        std::string ld;
+                        if (L.canvas_ld)
+                          ld = "P" + std::to_string(key.ring) + "_" + std::to_string(slot(key.ring, key.po)) + "[" +
+                               cbase(rc, RR.px) + " + " + std::to_string(key.off) + "]";
+                        else
+                          ld = "(ca" + rs + " && cx" + rs + " >= " + std::to_string(rc[0]) + " && cx" + rs + " < " +
+                               std::to_string(rc[1]) + " && cy" + rs + " >= " + std::to_string(rc[2]) + " && cy" + rs + " < " +
+                               std::to_string(rc[3]) + ") ? " + acc + " : (real)0";
                         if (carry.count(key))
                           o << "      const real " << nm << " = cqv ? " << key_name("cq", key, rs) << " : (" << ld << ");\n";
                         else
@@ -611,17 +627,7 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
   // lanes (first point's canvas x, row) needing each pair load over the whole fast iteration, and
   // whether the load can be issued unpredicated (every address it can form lies in the rings)
   std::map<PK, Rect> pall;
-  auto pair_nopred = [&](const PK& pk) {
-    const auto& [ring, po, rel] = pk;
-    const Ring& RR = L.rings[ring];
-    const long long cxmin = -PSH, cxmax = 2LL * (cv.cwp - 1) - PSH;
-    // inside the slot being read (see the single-point canvas above)
-    const long long amin = (cxmin + rel) * p.es;
-    const long long amax = ((long long)(CH - 1) * RR.px + cxmax + rel + 2) * p.es;
-    if (getenv("KF_LD_ANYRING"))   // A/B only: the racy round-1 rule
-      return L.canvas_ld && RR.smem_off + amin >= 0 && RR.smem_off + (long long)(RR.slots - 1) * RR.plane_bytes + amax <= L.mbar_off;
-    return L.canvas_ld && amin >= 0 && amax <= RR.plane_bytes;
-  };
+  auto pair_nopred = [&](const PK&) { return L.canvas_ld != 0; };   // clamped loads (cbase)
   // z register queues of the pair canvas: a pair value (ring, po, rel) read at iteration t is the
   // value (ring, po + 1, rel) had at iteration t - 1 -- loaded then by the same thread, or computed
   // then by it (its own forwarded result one plane earlier).  Such values are carried in registers
@@ -647,14 +653,16 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
             }
           }
     if (L.pair_zq)
-      for (auto& [pk, rc] : pall) {
+      for (auto& [pk, rc] : pall) {   // ascending (ring, plane offset): widening propagates upward
         const auto& [ring, po, rel] = pk;
         const PK nx{ring, po + 1, rel};
         auto it = pall.find(nx);
         if (it != pall.end()) {
-          const Rect& a = it->second;
-          const bool covers = pair_nopred(nx) || (a[0] <= rc[0] && a[1] >= rc[1] && a[2] <= rc[2] && a[3] >= rc[3]);
-          if (covers) pcarry[pk] = PSrc{true, nx, 0, 0};
+          // the source load must give every lane of this key's rectangle its true value: widen the
+          // source's lanes to the union (both lie in the ring box at every plane)
+          auto& a = it->second;
+          a = {std::min(a[0], rc[0]), std::max(a[1], rc[1]), std::min(a[2], rc[2]), std::max(a[3], rc[3])};
+          pcarry[pk] = PSrc{true, nx, 0, 0};
           continue;
         }
         // the thread's own result one plane earlier: an in-group ring, the pair of the thread's own
@@ -674,10 +682,11 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
     return "pq" + std::to_string(ring) + "_" + (po < 0 ? "m" + std::to_string(-po) : std::to_string(po)) + "_" +
            (rel < 0 ? "m" + std::to_string(-rel) : std::to_string(rel));
   };
-  auto pair_acc = [&](const PK& pk) {
+  auto pair_acc = [&](const PK& pk) {   // canvas_ld: the clamped base of the key's lanes (pall)
     const auto& [ring, po, rel] = pk;
-    return "*(const real2*)&P" + std::to_string(ring) + "_" + std::to_string(slot(ring, po)) + "[cb" +
-           std::to_string(L.rings[ring].px) + "_r0 + " + std::to_string(rel) + "]";
+    const std::string b = L.canvas_ld ? cbase(pall.at(pk), L.rings[ring].px) : "cb" + std::to_string(L.rings[ring].px) + "_r0";
+    return "*(const real2*)&P" + std::to_string(ring) + "_" + std::to_string(slot(ring, po)) + "[" + b + " + " +
+           std::to_string(rel) + "]";
   };
   auto pair_pred = [&](const Rect& rc) {
     return "ca_r0 && cx_r0 >= " + std::to_string(rc[0]) + " && cx_r0 < " + std::to_string(rc[1]) + " && cy_r0 >= " +
@@ -766,7 +775,7 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
                   auto it = ldname.find(pk);
                   if (it == ldname.end()) {
                     const auto& [ring, po, rel] = pk;
-                    const Rect& rc = prect.at(pk);
+                    const Rect& rc = pall.at(pk);   // (widened for z-queue carries)
                     const std::string nm = "pl" + std::to_string(ring) + "_" + (po < 0 ? "m" + std::to_string(-po) : std::to_string(po)) +
                                            "_" + (rel < 0 ? "m" + std::to_string(-rel) : std::to_string(rel)) + "_h" + std::to_string(ph);
                     const int mask = pmask.at(pk);
@@ -778,8 +787,10 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
                           << " : real2{(real)0, (real)0};\n";
                     } else {
                       const int c1 = mask == 2 ? 1 : 0;
-                      const std::string acc1 = "P" + std::to_string(ring) + "_" + std::to_string(slot(ring, po)) + "[cb" +
-                                               std::to_string(L.rings[ring].px) + "_r0 + " + std::to_string(rel + c1) + "]";
+                      const std::string b1 = L.canvas_ld ? cbase(pall.at(pk), L.rings[ring].px)
+                                                         : "cb" + std::to_string(L.rings[ring].px) + "_r0";
+                      const std::string acc1 = "P" + std::to_string(ring) + "_" + std::to_string(slot(ring, po)) + "[" + b1 + " + " +
+                                               std::to_string(rel + c1) + "]";
                       if (pair_nopred(pk)) o << "      const real " << nm << " = " << acc1 << ";\n";
                       else o << "      const real " << nm << " = (" << pair_pred(rc) << ") ? " << acc1 << " : (real)0;\n";
                     }
@@ -1405,6 +1416,11 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
   }
   o << "}\n";
   cg.source = o.str();
+  {
+    const std::string mark = "/*@@KF_CLAMP_BASES@@*/";
+    const size_t at = cg.source.find(mark);
+    if (at != std::string::npos) cg.source.replace(at, mark.size(), clamp_defs);
+  }
   return cg;
 }
 

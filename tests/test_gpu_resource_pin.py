@@ -60,7 +60,7 @@ def test_resource_model_bounds_loaded_kernels(cfg):
     for plan in plans:
         for cand in bench.AUTOTUNE_CANDIDATES:
             kw = bench.cand_kw(base, cand)
-            kw["ghostwrite"] = 1
+            kw["ghostwrite"] = 0
             jobs.append((plan, kw))
 
     def make(job):

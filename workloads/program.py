@@ -203,3 +203,15 @@ def footprint_radius(prog: Program) -> Tuple[int, int, int]:
                 for a in range(3):
                     r[a] = max(r[a], abs(d[a]))
     return tuple(r)
+
+
+def unroll(prog: Program, steps: int) -> Program:
+    """Temporal unrolling (NEXT-4, the temporal blocking of [15] cited at P:107 / P:556): the
+    description of `steps` consecutive timesteps as ONE step -- the kernel list repeated `steps`
+    times in order over the same arrays (kernel names suffixed with the sub-step).  Running the
+    result for N steps is, by definition, running `prog` for N*steps steps; a fusion plan of it may
+    group kernels of consecutive timesteps.  Pure description (no arithmetic of the method)."""
+    assert steps >= 1
+    kernels = [Kernel(f"{k.name}@{s}", [Stmt(st.out, list(st.rpn)) for st in k.stmts])
+               for s in range(steps) for k in prog.kernels]
+    return prog.with_(name=prog.name if steps == 1 else f"{prog.name}x{steps}", kernels=kernels)
