@@ -582,6 +582,11 @@ def run_kf(args):
     desc = wl.desc
     if args.relax_all and desc.name == "weather":
         desc = wl.desc = desc.with_(flags=PROG_RELAX_ALL)
+    S = max(1, args.unroll)
+    if S > 1:   # NEXT-4: S timesteps as one step of the unrolled program (plans may fuse across steps)
+        from workloads.program import unroll
+        desc = wl.desc = unroll(desc, S)
+        wl.label += f", unrolled x{S} (temporal fusion: one step = {S} timesteps)"
     tkw = dict(wl.tkw)
     if args.tile:
         tkw["tile"] = tuple(int(v) for v in args.tile.split(","))
@@ -697,12 +702,12 @@ def run_kf(args):
             d2h = sum(host[x].numel() * host[x].element_size() for x in outs)
             how = "kf.Dist.run with pinned host buffers copied in/out every step, host wall clock"
         dt = max_over_ranks(dt)
-        e2e = {"value": wl.global_npts * k / dt, "unit": UNIT, "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+        e2e = {"value": wl.global_npts * k * S / dt, "unit": UNIT, "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
                "steps": k, "timing": how + ", max over ranks"}
         del host
 
     bytes_step = info.compulsory_bytes_per_step
-    value = wl.global_npts * args.steps / (ms / 1e3)
+    value = wl.global_npts * args.steps * S / (ms / 1e3)
     peaks = measured_peaks()
     hbm_peak = peaks["hbm_gbs"] if peaks and "hbm_gbs" in peaks else 6650.0
     peak_src = "MEASURED_PEAKS.json hbm_gbs (burst copy)" if peaks else "B200_PROFILING.md fallback 6.65 TB/s"
@@ -749,7 +754,7 @@ def run_kf(args):
     px, py = grid_for(world)
     res = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
-        "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": wl.scaling, "vs_baseline": None,
+        "ms_per_step": ms / args.steps / S, "higher_is_better": True, "scaling": wl.scaling, "vs_baseline": None,
         "dtype": "f64" if desc.dtype == 1 else "f32", "data": "synthetic (seeded, paper-shaped fields)",
         "config": {"workload": wl.label + (" with RELAX_ALL renaming" if desc.flags & 2 else ""),
                    "plan": f"{plan_kind}: {info.n_groups} fused groups of {prog.nk} kernels",
@@ -895,6 +900,7 @@ def main():
                     help="select: measured choice among the searches' candidates; best: HGGA/brute on projected "
                          "time; unfused; hand; or a JSON label list (config.plan_labels of an earlier run)")
     ap.add_argument("--relax-all", type=int, default=0, help="weather: rename every written array (KF_PROG_RELAX_ALL)")
+    ap.add_argument("--unroll", type=int, default=1, help="NEXT-4 temporal fusion: plan over S timesteps as one step")
     ap.add_argument("--tile", default=None)
     ap.add_argument("--stages", type=int, default=None)
     ap.add_argument("--threads", type=int, default=None)

@@ -6,6 +6,7 @@
 //   base + (k+gz)*plane + (j+gy)*pitch + xoff + i.
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 
 #include "kf_kernels.hpp"
 
@@ -104,6 +105,59 @@ __global__ void fill_xy_multi(FillList L, Geom g, int px, int py, int frozen_onl
   }
 }
 
+// Periodic x and y ghosts of several buffers in one launch (blockIdx.y = buffer), written in whole
+// 32-byte sectors: a ghost span is widened to sector boundaries (padding cells take any wrapped
+// value; an interior cell in a shared sector is rewritten with itself), so no store is a partial
+// sector (a partial sector costs the L2 a read-modify-write with ECC; measured round 2).  Lanes map
+// to consecutive cells of a row span, so a warp stores whole sectors.  Every written cell takes the
+// interior cell its coordinates wrap to on the periodic axes (corners included), as fill_xy_multi.
+// Pieces: x spans of every row (x periodic; interior rows only if y is periodic as well), then
+// whole y-ghost rows (y periodic).  frozen_only (bits x/y/z frozen): only cells inside a frozen
+// axis' ghost layer, exact cells (the run-start fill of scratch buffers).
+template <typename T>
+__global__ void fill_xy_sectors(FillList L, Geom g, int px, int py, int frozen_only) {
+  T* base = (T*)L.base[blockIdx.y];
+  constexpr int E = 32 / sizeof(T);
+  const int NZ = g.nz + 2 * g.gz;
+  const int xl0 = -((g.gx + E - 1) / E) * E;                 // left span [xl0, 0)
+  const int xr0 = (g.nx / E) * E, xr1 = ((g.nx + g.gx + E - 1) / E) * E;   // right span [xr0, xr1)
+  const int cx = px ? (-xl0) + (xr1 - xr0) : 0;              // cells per row of the x pass
+  const int rows_x = py ? g.ny : g.ny + 2 * g.gy;
+  const int jx0 = py ? 0 : -g.gy;
+  const int cy = py ? xr1 - xl0 : 0;                         // cells per y-ghost row: [xl0, xr1)
+  const long long nx_cells = (long long)cx * rows_x * NZ, ny_cells = (long long)cy * 2 * g.gy * NZ;
+  for (long long idx = blockIdx.x * (long long)blockDim.x + threadIdx.x; idx < nx_cells + ny_cells;
+       idx += (long long)gridDim.x * blockDim.x) {
+    int i, j, k;
+    if (idx < nx_cells) {
+      const unsigned q = unsigned(idx);
+      const unsigned r = q / unsigned(cx), c = q - r * unsigned(cx);
+      k = int(r / unsigned(rows_x)) - g.gz;
+      j = jx0 + int(r % unsigned(rows_x));
+      i = int(c) < -xl0 ? xl0 + int(c) : xr0 + int(c) + xl0;
+    } else {
+      const unsigned q = unsigned(idx - nx_cells);
+      const unsigned r = q / unsigned(cy), c = q - r * unsigned(cy);
+      const int e = int(r % unsigned(2 * g.gy));
+      k = int(r / unsigned(2 * g.gy)) - g.gz;
+      j = e < g.gy ? -1 - e : g.ny + (e - g.gy);
+      i = xl0 + int(c);
+    }
+    if (frozen_only) {
+      const bool gi = i < 0 || i >= g.nx, gj = j < 0 || j >= g.ny, gk = k < 0 || k >= g.nz;
+      const bool cell = (px ? (i >= -g.gx && i < g.nx + g.gx) : true) && (py ? (j >= -g.gy && j < g.ny + g.gy) : true);
+      if (!cell || (!gi && !gj) || !(((frozen_only & 1) && gi) || ((frozen_only & 2) && gj) || ((frozen_only & 4) && gk)))
+        continue;
+    }
+    int si = i, sj = j;
+    if (px && (i < 0 || i >= g.nx)) si = ((i % g.nx) + g.nx) % g.nx;
+    if (!px) si = i < -g.gx ? -g.gx : (i >= g.nx + g.gx ? g.nx + g.gx - 1 : i);   // padding: any stored cell
+    if (py && (j < 0 || j >= g.ny)) sj = ((j % g.ny) + g.ny) % g.ny;
+    const long long o = (long long)(k + g.gz) * g.plane + g.xoff;
+    base[o + (long long)(j + g.gy) * g.pitch + i] = base[o + (long long)(sj + g.gy) * g.pitch + si];
+  }
+}
+
 // Copy every element that is not interior (ghost shell and padding) from src to dst:
 // renamed copies of an array share its frozen ghost values (R9).
 template <typename T>
@@ -182,8 +236,17 @@ cudaError_t launch_fill_xy_multi(void* const* bufs, int n, int px, int py, int e
                                  int frozen_only) {
   if (!px && !py) return cudaSuccess;
   const long long NZ = g.nz + 2 * g.gz;
-  const long long per = (px ? 2LL * g.gx * (g.ny + 2 * g.gy) : 0) * NZ +
-                        (py ? (long long)(px ? g.nx : g.nx + 2 * g.gx) * 2 * g.gy * NZ : 0);
+  // sector-wide writes need the row origin (x = 0) 32-byte aligned (kf_array_layout: 128-byte rows)
+  const int E = 32 / es;
+  const bool sectors = !getenv("KF_FILL_CELLS") && (g.xoff * (long long)es) % 32 == 0 && (g.pitch * (long long)es) % 32 == 0 &&
+                       (g.plane * (long long)es) % 32 == 0 && ((g.gx + E - 1) / E) * E <= g.xoff;
+  long long per = (px ? 2LL * g.gx * (g.ny + 2 * g.gy) : 0) * NZ +
+                  (py ? (long long)(px ? g.nx : g.nx + 2 * g.gx) * 2 * g.gy * NZ : 0);
+  if (sectors) {
+    const long long xl = ((g.gx + E - 1) / E) * E, xr = ((g.nx + g.gx + E - 1) / E) * E - (g.nx / E) * E;
+    per = (px ? (xl + xr) * (long long)(py ? g.ny : g.ny + 2 * g.gy) : 0) * NZ +
+          (py ? (xl + (long long)((g.nx + g.gx + E - 1) / E) * E) * 2 * g.gy * NZ : 0);
+  }
   if (per == 0) return cudaSuccess;
   for (int b0 = 0; b0 < n; b0 += kMaxFillBufs) {
     const int m = n - b0 < kMaxFillBufs ? n - b0 : kMaxFillBufs;
@@ -192,7 +255,9 @@ cudaError_t launch_fill_xy_multi(void* const* bufs, int n, int px, int py, int e
     long long nb = (per + 255) / 256;
     const long long cap = (148LL * 16 + m - 1) / m;   // ~16 CTAs per SM over all buffers
     dim3 grid(unsigned(nb < cap ? nb : cap), unsigned(m));
-    if (es == 4) fill_xy_multi<float><<<grid, 256, 0, s>>>(L, g, px, py, frozen_only);
+    if (sectors && es == 4) fill_xy_sectors<float><<<grid, 256, 0, s>>>(L, g, px, py, frozen_only);
+    else if (sectors) fill_xy_sectors<double><<<grid, 256, 0, s>>>(L, g, px, py, frozen_only);
+    else if (es == 4) fill_xy_multi<float><<<grid, 256, 0, s>>>(L, g, px, py, frozen_only);
     else fill_xy_multi<double><<<grid, 256, 0, s>>>(L, g, px, py, frozen_only);
   }
   return cudaGetLastError();
