@@ -322,9 +322,10 @@ typedef struct {
 } kf_exec_info;
 kf_status kf_exec_get_info(const kf_exec* ex, kf_exec_info* out);
 /* Per-group launch details: grid, threads, dynamic SMEM, registers (cuFuncGetAttribute),
- * local (spill) bytes, compulsory bytes per launch, kernel name.  name: >= 64 chars. */
+ * local (spill) bytes, the loaded function's maximum threads per CTA (-1 before loading),
+ * compulsory bytes per launch, kernel name.  name: >= 64 chars. */
 typedef struct {
-  int32_t group, grid, threads, smem_bytes, regs, local_bytes, n_kernels, pad;
+  int32_t group, grid, threads, smem_bytes, regs, local_bytes, n_kernels, max_threads;
   uint64_t bytes_per_launch;
   char name[64];
 } kf_group_info;

@@ -279,7 +279,7 @@ def schedule(prog: Program, grp: List[int], target: Target):
         kmax = max(kmax, nk)
     thrld = len(loads) if canvas else kmax
     regs = 32 * target.zunroll + (es // 4) * P * (thrld + depth)
-    return dict(ext=ext, pts=pts, delay=D, res=res, smem=smem, regs=regs, alive=alive)
+    return dict(ext=ext, pts=pts, delay=D, res=res, smem=smem, regs=regs, alive=alive, threads=threads)
 
 
 # ---------------------------------------------------------------- validation
@@ -385,8 +385,8 @@ def validate(prog: Program, plan: List[int], target: Target = Target()):
     for g in range(m):
         if scheds[g]["smem"] > target.smem_per_block:
             return (V7_SMEM, g, -1, -1, -1)
-    for g in range(m):
-        if scheds[g]["regs"] > target.regs_per_thread_max:
+    for g in range(m):   # Eq. 2 (R_T <= R_Max) and Eq. 3 with one CTA per SM (Thr * R_T <= R_SMX = 65536)
+        if scheds[g]["regs"] > target.regs_per_thread_max or scheds[g]["regs"] * scheds[g]["threads"] > 65536:
             return (V8_REGS, g, -1, -1, -1)
     return NONE
 

@@ -144,23 +144,28 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
   // register cap (__maxnreg__): at most what keeps the shared-memory-limited number of CTAs per SM
   // resident (minblocks 0; or minblocks CTAs) and never above the resource model's estimate R_est
   // (V8, R20).  The runtime recompiles without the cap if it would make ptxas spill.
-  // Registers.  minblocks -1: __launch_bounds__(NT), ptxas' own choice -- the register model R_est
-  // (V8) must bound it; a GPU test pins NUM_REGS <= R_est and no spills over every bench
-  // configuration.  (Measured: explicit budgets -- __maxnreg__(R_est), or __launch_bounds__ with a
-  // minimum CTA count -- make ptxas use up to the budget, e.g. 124 or 162 instead of 88 or 72
-  // registers on the flux groups, one CTA per SM less.)  minblocks >= 0: __maxnreg__ keeps the
-  // shared-memory-limited number of CTAs per SM resident (0) or n CTAs (n >= 1), never above R_est;
-  // if that would make ptxas spill, the runtime rebuilds without it (KF_NO_MAXNREG).
-  if (const char* fc = getenv("KF_MAXNREG")) {   // experiments only: force a register cap
-    o << "#define KF_BOUNDS __maxnreg__(" << atoi(fc) << ")\n";
-  } else if (L.minblocks >= 0) {
-    const int smem_ctas = 233472 / std::max(1, L.smem + 1024);
-    const int minb = L.minblocks > 0 ? L.minblocks : std::max(1, std::min({smem_ctas, 2048 / std::max(1, NT), 8}));
-    const int cap = std::max(24, std::min({65536 / (NT * minb) / 8 * 8, L.regs, 255}));
-    o << "#ifndef KF_NO_MAXNREG\n#define KF_BOUNDS __maxnreg__(" << cap
-      << ")\n#else\n#define KF_BOUNDS __launch_bounds__(NT)\n#endif\n";
-  } else {
-    o << "#define KF_BOUNDS __launch_bounds__(NT)\n";
+  // Registers.  minblocks -1: __launch_bounds__(NT), ptxas' own choice (measured: explicit budgets
+  // make ptxas use up to the budget, e.g. 124 or 162 instead of 88 or 72 registers on the flux
+  // groups, one CTA per SM less); minblocks >= 0: __maxnreg__ keeps the shared-memory-limited number
+  // of CTAs per SM resident (0) or n CTAs (n >= 1), never above R_est.  Fallback (KF_NO_MAXNREG),
+  // compiled when the first build spills or uses more registers than the register model R_est
+  // (V8): __maxnreg__(R_est) (and no more than NT threads allow).  So the loaded kernel never has
+  // more than R_est registers; a GPU test pins that it does not spill either.
+  {
+    const int rest = std::max(24, std::min({L.regs, 255, 65536 / std::max(1, NT) / 8 * 8}));
+    std::string primary;
+    if (const char* fc = getenv("KF_MAXNREG")) {   // experiments only: force a register cap
+      primary = "__maxnreg__(" + std::to_string(atoi(fc)) + ")";
+    } else if (L.minblocks >= 0) {
+      const int smem_ctas = 233472 / std::max(1, L.smem + 1024);
+      const int minb = L.minblocks > 0 ? L.minblocks : std::max(1, std::min({smem_ctas, 2048 / std::max(1, NT), 8}));
+      const int cap = std::max(24, std::min(65536 / (NT * minb) / 8 * 8, rest));
+      primary = "__maxnreg__(" + std::to_string(cap) + ")";
+    } else {
+      primary = "__launch_bounds__(NT)";
+    }
+    o << "#define KF_REST " << rest << "\n#ifndef KF_NO_MAXNREG\n#define KF_BOUNDS " << primary
+      << "\n#else\n#define KF_BOUNDS __maxnreg__(KF_REST)\n#endif\n";
   }
   o << "extern \"C\" __global__ void KF_BOUNDS " << cg.name << "(const __grid_constant__ KfArgs a) {\n";
   // pointer arithmetic from the __shared__ array keeps the shared state space (LDS/STS, 32-bit
@@ -232,7 +237,7 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
     auto it = clamp_base.find(key);
     if (it != clamp_base.end()) return it->second;
     const std::string nm = "ckb" + std::to_string(clamp_base.size());
-    const std::string cy = "min(max(cy_r0, " + std::to_string(rc[2]) + "), " + std::to_string(rc[3] - 1) + ")";
+    const std::string cy = "min(max(cy_r0 + kz, " + std::to_string(rc[2]) + "), " + std::to_string(rc[3] - 1) + ")";
     std::string cx;
     if (pair_mode) {   // first-point x of an aligned pair inside [x0, x1): pair columns [lo, hi]
       const int lo = (rc[0] + PSH + 1) >> 1, hi = (rc[1] - 1 + PSH) >> 1;
@@ -240,7 +245,7 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
     } else {
       cx = "min(max(cx_r0, " + std::to_string(rc[0]) + "), " + std::to_string(rc[1] - 1) + ")";
     }
-    clamp_defs += "  const int " + nm + " = " + cy + " * " + std::to_string(pitch) + " + " + cx + ";\n";
+    clamp_defs += "      const int " + nm + " = " + cy + " * " + std::to_string(pitch) + " + " + cx + ";\n";
     clamp_base.emplace(key, nm);
     return nm;
   };
@@ -298,7 +303,6 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
           << " && cy" << rs << " >= " << oy << " && cy" << rs << " < " << oy + WY << ";\n";
       }
     }
-  o << "/*@@KF_CLAMP_BASES@@*/";
   o << "  __syncthreads();\n";
   // per-kernel compute / ghost plane ranges for this unit
   for (int k : alive) {
@@ -1286,6 +1290,9 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
     }
     if (!getenv("KF_CANVAS_COND")) c = "t >= cf0 && t < cf1";   // A/B switch: the per-kernel conjunction
     o << "    if (" << c << ") {   // ---- fast iteration on the canvas\n";
+    // clamped load bases (canvas_ld), recomputed every iteration from an opaque zero so the compiler
+    // does not keep them live across the stream loop (cheap integer ops instead of registers)
+    o << "      int kz;\n      asm volatile(\"mov.u32 %0, 0;\" : \"=r\"(kz));\n/*@@KF_CLAMP_BASES@@*/";
     if (pair_mode) emit_canvas_pairs();
     else emit_canvas();
     o << "    } else {\n";
@@ -1418,8 +1425,8 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
   cg.source = o.str();
   {
     const std::string mark = "/*@@KF_CLAMP_BASES@@*/";
-    const size_t at = cg.source.find(mark);
-    if (at != std::string::npos) cg.source.replace(at, mark.size(), clamp_defs);
+    for (size_t at = cg.source.find(mark); at != std::string::npos; at = cg.source.find(mark, at))
+      cg.source.replace(at, mark.size(), clamp_defs);
   }
   return cg;
 }

@@ -433,6 +433,11 @@ bool quotient_acyclic(const Program& p, const std::vector<int>& label, int m, in
   return true;
 }
 
+// V8 = Eq. 2 (R_T <= R_Max) and Eq. 3 with one CTA per SM (Thr * R_T <= R_SMX = 65536 on B200)
+bool regs_ok(const GroupLowering& L, const kf_target& t) {
+  return L.regs <= t.regs_per_thread_max && int64_t(L.regs) * L.threads <= 65536;
+}
+
 int validate_plan_groups(const Program& p, const Plan& pl, const std::vector<kf_target>& T, kf_violation* why,
                          std::vector<GroupLowering>* lowered) {
   if (why) *why = kf_violation{KF_V_OK, -1, -1, -1, -1};
@@ -458,7 +463,7 @@ int validate_plan_groups(const Program& p, const Plan& pl, const std::vector<kf_
       return KF_V_SMEM;
     }
   for (int gi = 0; gi < pl.m; gi++)
-    if (Ls[gi].regs > T[gi].regs_per_thread_max) {
+    if (!regs_ok(Ls[gi], T[gi])) {
       if (why) *why = kf_violation{KF_V_REGS, gi, -1, -1, -1};
       return KF_V_REGS;
     }

@@ -38,10 +38,15 @@ struct Drv {
   CUresult (*getErrorString)(CUresult, const char**) = nullptr;
 };
 
+// (a failing runtime call also leaves its error as the thread's "last error": clear it, or the next
+// launch helper's cudaGetLastError() would report it again)
 #define CK(x)                                                                                       \
   do {                                                                                              \
     cudaError_t e_ = (x);                                                                           \
-    if (e_ != cudaSuccess) fail(KF_E_CUDA, std::string(#x) + ": " + cudaGetErrorString(e_));        \
+    if (e_ != cudaSuccess) {                                                                        \
+      cudaGetLastError();                                                                           \
+      fail(KF_E_CUDA, std::string(#x) + ": " + cudaGetErrorString(e_));                             \
+    }                                                                                               \
   } while (0)
 
 static Drv& drv() {
@@ -80,7 +85,7 @@ struct Compiled {
   std::vector<char> cubin;
   std::string log;
   int regs_ptxas = -1, spill = -1;
-  bool nocap = false;   // compiled with KF_NO_MAXNREG (occupancy register cap dropped)
+  bool nocap = false;   // compiled with KF_NO_MAXNREG (the fallback build at __maxnreg__(R_est))
 };
 
 static Compiled nvrtc_compile(const std::string& src, const std::string& name) {
@@ -127,6 +132,12 @@ static Compiled nvrtc_compile(const std::string& src, const std::string& name) {
 static std::mutex g_cache_mu;
 static std::map<std::string, std::shared_ptr<Compiled>> g_cubin_cache;   // source -> cubin
 
+// register model bound the kernel was generated for (#define KF_REST n)
+static int source_rest(const std::string& src) {
+  const auto p = src.find("#define KF_REST ");
+  return p == std::string::npos ? 255 : atoi(src.c_str() + p + 16);
+}
+
 static std::shared_ptr<Compiled> compile_cached(const std::string& src, const std::string& name) {
   {
     std::lock_guard<std::mutex> lk(g_cache_mu);
@@ -134,8 +145,9 @@ static std::shared_ptr<Compiled> compile_cached(const std::string& src, const st
     if (it != g_cubin_cache.end()) return it->second;
   }
   auto c = std::make_shared<Compiled>(nvrtc_compile(src, name));
-  // the occupancy register cap (__maxnreg__) must not cost local-memory spills: rebuild without it
-  if (c->spill > 0 && src.find("#ifndef KF_NO_MAXNREG") != std::string::npos) {
+  // the first build must neither spill nor exceed the register model (V8): else the fallback build
+  // at __maxnreg__(R_est)
+  if ((c->spill > 0 || c->regs_ptxas > source_rest(src)) && src.find("#ifndef KF_NO_MAXNREG") != std::string::npos) {
     c = std::make_shared<Compiled>(nvrtc_compile("#define KF_NO_MAXNREG 1\n" + src, name));
     c->nocap = true;
   }
@@ -174,7 +186,7 @@ struct GroupExec {
   std::shared_ptr<Compiled> comp;
   CUmodule mod = nullptr;
   CUfunction fn = nullptr;
-  int grid = 0, smem = 0, regs = -1, local = -1;
+  int grid = 0, smem = 0, regs = -1, local = -1, maxthr = -1;
   Split split;   // interior / boundary units (a11 overlap)
   uint64_t bytes = 0;
   std::vector<Ver> ins, outs, mids;
@@ -359,6 +371,9 @@ static void launch_group(kf_exec* E, int gi, int par, cudaStream_t s, int mode =
     for (size_t i = 0; i < blob.size(); i += 8) fprintf(stderr, " %016llx", *(unsigned long long*)(tmp + i));
     fprintf(stderr, "\n");
   }
+  if (g.maxthr > 0 && g.L.threads > g.maxthr)
+    fail(KF_E_RESOURCE, g.cg.name + ": " + std::to_string(g.L.threads) + " threads per CTA but the compiled kernel allows " +
+                            std::to_string(g.maxthr) + " (" + std::to_string(g.regs) + " registers)");
   ckd(drv().launchKernel(g.fn, grid, 1, 1, g.L.threads, 1, 1, g.smem, (CUstream)s, params, nullptr),
       ("cuLaunchKernel " + g.cg.name).c_str());
 }
@@ -433,8 +448,10 @@ static void ensure_device(kf_exec* E) {
           "cuFuncSetAttribute(MAX_DYNAMIC_SHARED_SIZE_BYTES)");
       drv().funcGetAttribute(&g.regs, CU_FUNC_ATTRIBUTE_NUM_REGS, g.fn);
       drv().funcGetAttribute(&g.local, CU_FUNC_ATTRIBUTE_LOCAL_SIZE_BYTES, g.fn);
+      drv().funcGetAttribute(&g.maxthr, CU_FUNC_ATTRIBUTE_MAX_THREADS_PER_BLOCK, g.fn);
       // the register cap must not cost local memory (spills): rebuild without it
-      if (g.local > 0 && !g.comp->nocap && g.cg.source.find("#ifndef KF_NO_MAXNREG") != std::string::npos) {
+      if ((g.local > 0 || g.regs > source_rest(g.cg.source)) && !g.comp->nocap &&
+          g.cg.source.find("#ifndef KF_NO_MAXNREG") != std::string::npos) {
         g.comp = compile_nocap(g.cg.source, g.cg.name);
         if (drv().moduleUnload) drv().moduleUnload(g.mod);
         g.mod = nullptr;
@@ -810,6 +827,7 @@ kf_status kf_exec_group_info(const kf_exec* ex, int32_t group, kf_group_info* ou
     r.regs = g.regs >= 0 ? g.regs : g.comp->regs_ptxas;
     r.local_bytes = g.local >= 0 ? g.local : g.comp->spill;
     r.n_kernels = int(g.L.kernels.size());
+    r.max_threads = g.maxthr;
     r.bytes_per_launch = g.bytes;
     std::strncpy(r.name, g.cg.name.c_str(), sizeof(r.name) - 1);
     *out = r;

@@ -38,7 +38,7 @@ class Evaluator {
     } else {
       GroupLowering L = lower_group(p_, g, t_);
       if (check_hazard(p_, g, L, 0, nullptr) || check_halo(p_, L, t_, 0, nullptr) || L.smem > t_.smem_per_block ||
-          L.regs > t_.regs_per_thread_max)
+          !regs_ok(L, t_))
         v.ok = false;
       else
         v.t_model = model_time(p_, L, t_, v.bytes);

@@ -33,11 +33,11 @@ def main():
         desc = P.weather(n=(64, 48, 12))
         inputs = D.weather_inputs(desc, 3)
         prog0 = kf.Program(desc)
-        plan, _ = prog0.search(kf.SEARCH_HGGA, kf.Target(tile=(32, 8, 0)), seed=1)
         if mode == "pairs":
             tgt = kf.Target(tile=(32, 8, 0), pblock=(2, 1), pair_zq=1, canvas_ld=1, minblocks=-1)
         else:
             tgt = kf.Target(tile=(32, 8, 0), pblock=(1, 1), canvas_ld=1, minblocks=-1)
+        plan, _ = prog0.search(kf.SEARCH_HGGA, tgt, seed=1)   # legal under this launch configuration (V8)
     prog = kf.Program(desc)
     ex = kf.Exec(prog, plan, tgt)
     ex.set_graph(False)
