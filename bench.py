@@ -584,7 +584,10 @@ def run_kf(args):
         desc = wl.desc = desc.with_(flags=PROG_RELAX_ALL)
     S = max(1, args.unroll)
     if S > 1:   # NEXT-4: S timesteps as one step of the unrolled program (plans may fuse across steps)
+        from workloads import programs
         from workloads.program import unroll
+        if desc.name == "weather":   # cross-step fusion accumulates halos: a deeper periodic ghost (V6)
+            desc = programs.weather(n=desc.n, ghost=(2 * S, 2 * S, 2), relax=desc.flags)
         desc = wl.desc = unroll(desc, S)
         wl.label += f", unrolled x{S} (temporal fusion: one step = {S} timesteps)"
     tkw = dict(wl.tkw)

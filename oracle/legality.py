@@ -282,6 +282,14 @@ def schedule(prog: Program, grp: List[int], target: Target):
     return dict(ext=ext, pts=pts, delay=D, res=res, smem=smem, regs=regs, alive=alive, threads=threads)
 
 
+def regs_limit(threads: int) -> int:
+    """Registers per thread an NT-thread CTA can have on B200 (Eq. 3 with one CTA per SM): the
+    65536-register file is 4 sub-partitions of 16384, a CTA's warps spread over them, allocation in
+    units of 8 registers per thread."""
+    warps = -(-threads // 32)
+    return min(255, 16384 // (-(-warps // 4) * 32) // 8 * 8)
+
+
 # ---------------------------------------------------------------- validation
 def quotient_order(prog: Program, plan: List[int]):
     """Kahn order of groups; ties -> smaller canonical label (smallest first kernel)."""
@@ -385,8 +393,8 @@ def validate(prog: Program, plan: List[int], target: Target = Target()):
     for g in range(m):
         if scheds[g]["smem"] > target.smem_per_block:
             return (V7_SMEM, g, -1, -1, -1)
-    for g in range(m):   # Eq. 2 (R_T <= R_Max) and Eq. 3 with one CTA per SM (Thr * R_T <= R_SMX = 65536)
-        if scheds[g]["regs"] > target.regs_per_thread_max or scheds[g]["regs"] * scheds[g]["threads"] > 65536:
+    for g in range(m):   # Eq. 2 (R_T <= R_Max) and Eq. 3 with one CTA per SM (per register-file quadrant)
+        if scheds[g]["regs"] > min(target.regs_per_thread_max, regs_limit(scheds[g]["threads"])):
             return (V8_REGS, g, -1, -1, -1)
     return NONE
 

@@ -152,14 +152,14 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
   // (V8): __maxnreg__(R_est) (and no more than NT threads allow).  So the loaded kernel never has
   // more than R_est registers; a GPU test pins that it does not spill either.
   {
-    const int rest = std::max(24, std::min({L.regs, 255, 65536 / std::max(1, NT) / 8 * 8}));
+    const int rest = std::max(24, std::min(L.regs, regs_limit(NT)));
     std::string primary;
     if (const char* fc = getenv("KF_MAXNREG")) {   // experiments only: force a register cap
       primary = "__maxnreg__(" + std::to_string(atoi(fc)) + ")";
     } else if (L.minblocks >= 0) {
       const int smem_ctas = 233472 / std::max(1, L.smem + 1024);
       const int minb = L.minblocks > 0 ? L.minblocks : std::max(1, std::min({smem_ctas, 2048 / std::max(1, NT), 8}));
-      const int cap = std::max(24, std::min(65536 / (NT * minb) / 8 * 8, rest));
+      const int cap = std::max(24, std::min(regs_limit(NT * minb), rest));
       primary = "__maxnreg__(" + std::to_string(cap) + ")";
     } else {
       primary = "__launch_bounds__(NT)";

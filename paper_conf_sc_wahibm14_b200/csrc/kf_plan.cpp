@@ -433,9 +433,19 @@ bool quotient_acyclic(const Program& p, const std::vector<int>& label, int m, in
   return true;
 }
 
-// V8 = Eq. 2 (R_T <= R_Max) and Eq. 3 with one CTA per SM (Thr * R_T <= R_SMX = 65536 on B200)
+// Registers a thread of an NT-thread CTA can have: the register file is 4 sub-partitions of 16384
+// (B200: 65536 per SM), a CTA's warps spread over them round-robin, allocation in units of 8
+// registers per thread (256 per warp) -- measured: a 320-thread kernel at 192 registers reports
+// CU_FUNC_ATTRIBUTE_MAX_THREADS_PER_BLOCK = 256.
+int regs_limit(int threads) {
+  const int warps = (threads + 31) / 32;
+  const int per_quadrant = (warps + 3) / 4;
+  return std::min(255, 16384 / (per_quadrant * 32) / 8 * 8);
+}
+
+// V8 = Eq. 2 (R_T <= R_Max) and Eq. 3 with one CTA per SM (Thr * R_T <= R_SMX, per sub-partition)
 bool regs_ok(const GroupLowering& L, const kf_target& t) {
-  return L.regs <= t.regs_per_thread_max && int64_t(L.regs) * L.threads <= 65536;
+  return L.regs <= t.regs_per_thread_max && L.regs <= regs_limit(L.threads);
 }
 
 int validate_plan_groups(const Program& p, const Plan& pl, const std::vector<kf_target>& T, kf_violation* why,

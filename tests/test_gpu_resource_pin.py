@@ -80,7 +80,6 @@ def test_resource_model_bounds_loaded_kernels(cfg):
         if ex is None:
             # only V7/V8 (launch-configuration dependent) may reject a plan the search produced
             assert v[0] in (7, 8), (plan, kw, v)
-            assert v[0] != 8 or any(g.regs_est > 255 for g in per)
             rejected += 1
             continue
         ex.load()

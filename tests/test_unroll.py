@@ -24,7 +24,7 @@ def test_unrolled_step_equals_two_steps(which):
 
 def test_unrolled_weather_plans_cross_steps():
     kf = pytest.importorskip("paper_conf_sc_wahibm14_b200")
-    desc = P.weather(n=(64, 48, 12))
+    desc = P.weather(n=(64, 48, 12), ghost=(4, 4, 2))   # cross-step halos need a deeper periodic ghost (V6)
     u = unroll(desc, 2)
     prog = kf.Program(u)
     t = kf.Target(tile=(32, 8, 0))
