@@ -202,20 +202,35 @@ def select_plan(prog, target, dev, steps=5):
     launch configuration and timed (CUDA events, `steps` steps after 2 warm-up steps); the
     fastest is kept.  The projection ranks plans inside the search; the measurement decides
     between the few it proposes."""
+    import torch
     import paper_conf_sc_wahibm14_b200 as kf
     res = []
     for plan, kind in plan_candidates(prog, target):
         try:
             ex = kf.Exec(prog, plan, target)
         except Exception as e:   # an illegal candidate for this target: skip it
-            res.append((float("inf"), plan, kind + f" (failed: {str(e)[:80]})"))
+            res.append((float("inf"), plan, kind + f" (failed: {str(e)[:80]})", []))
             continue
-        res.append((time_exec(ex, dev, steps), plan, kind))
-        del ex
+        ms = time_exec(ex, dev, steps)
+        # per-group times of the candidate under the default launch configuration (NEXT-2 data:
+        # measured vs projected for every group the searches propose)
+        sb = ex.scratch_bytes()
+        scr = torch.empty(sb, dtype=torch.uint8, device="cuda") if sb else None
+        ex.set_profiling(True)
+        ex.run(dev, scr, steps)
+        torch.cuda.synchronize()
+        gms, _ = ex.group_times()
+        ex.set_profiling(False)
+        per, _, _ = prog.project(plan, target)
+        groups = [{"kernels": [k for k in range(len(plan)) if plan[k] == g], "ms": gms[g] / steps, "t_model_ms": per[g].t_model_s * 1e3,
+                   "t_bytes_ms": per[g].t_s * 1e3, "regs": ex.group_info(g).regs} for g in range(len(gms))]
+        res.append((ms, plan, kind, groups))
+        del ex, scr
     best = min(res, key=lambda r: r[0])
-    ranked = [(plan, kind) for ms, plan, kind in sorted(res, key=lambda r: r[0]) if ms < float("inf")]
+    ranked = [(plan, kind) for ms, plan, kind, _ in sorted(res, key=lambda r: r[0]) if ms < float("inf")]
     return best[1], best[2] + " (fastest of the measured candidates)", [
-        {"plan": kind, "ms_per_step": round(ms, 4), "groups": len(set(plan))} for ms, plan, kind in res], ranked
+        {"plan": kind, "ms_per_step": round(ms, 4), "groups": len(set(plan)), "labels": plan, "per_group": g}
+        for ms, plan, kind, g in res], ranked
 
 
 def choose_plan(prog, target, which: str):
