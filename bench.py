@@ -287,6 +287,10 @@ class ClockSampler:
         return self
 
     def mark_start(self):
+        # the sampler must be running before the timed region starts (short regions: tens of ms)
+        t_wait = time.perf_counter()
+        while self.h is not None and not self.samples and time.perf_counter() - t_wait < 1.0:
+            time.sleep(0.001)
         self.t0 = time.perf_counter()
 
     def mark_end(self):
@@ -303,7 +307,7 @@ class ClockSampler:
             except Exception as e:
                 self.err = f"{type(e).__name__}: {e}"
                 return
-            time.sleep(0.005)
+            time.sleep(0.002)
 
     def __exit__(self, *a):
         self.stop.set()
@@ -325,7 +329,7 @@ class ClockSampler:
                 if rs & getattr(self.nv, attr, 0):
                     reasons.add(nm)
         return {"sm_mhz": sm[len(sm) // 2], "sm_max_mhz": self.max_mhz, "reasons": sorted(reasons),
-                "samples": len(win), "source": "NVML, 5 ms, inside the timed region"}
+                "samples": len(win), "source": "NVML, every 2 ms, inside the timed region"}
 
 
 def measured_peaks():
