@@ -141,31 +141,40 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
   o << "  double prm[" << std::max(1, p.n_params) << "];\n";
   o << "  int mode, pad_;   // units: 0 all, 1 interior tiles only, 2 the others (kf_split_units)\n";
   o << "};\n";
-  // register cap (__maxnreg__): at most what keeps the shared-memory-limited number of CTAs per SM
-  // resident (minblocks 0; or minblocks CTAs) and never above the resource model's estimate R_est
-  // (V8, R20).  The runtime recompiles without the cap if it would make ptxas spill.
   // Registers.  minblocks -1: __launch_bounds__(NT), ptxas' own choice (measured: explicit budgets
   // make ptxas use up to the budget, e.g. 124 or 162 instead of 88 or 72 registers on the flux
-  // groups, one CTA per SM less); minblocks >= 0: __maxnreg__ keeps the shared-memory-limited number
-  // of CTAs per SM resident (0) or n CTAs (n >= 1), never above R_est.  Fallback (KF_NO_MAXNREG),
-  // compiled when the first build spills or uses more registers than the register model R_est
-  // (V8): __maxnreg__(R_est) (and no more than NT threads allow).  So the loaded kernel never has
-  // more than R_est registers; a GPU test pins that it does not spill either.
+  // groups, one CTA per SM less).  minblocks >= 0: __maxnreg__ at what keeps m CTAs per SM resident
+  // (m = the shared-memory-limited count for 0, n for n >= 1), never above R_est.  Register cliffs
+  // are steep (measured: 67 instead of 64 registers halved the CTAs per SM of a 448-thread group), so
+  // a build that spills steps down the ladder m-1, m-2, ... CTAs and finally R_est (V8): the runtime
+  // compiles "#define KF_CAP c" for the next cap of "// KF_CAPS" until ptxas neither spills nor
+  // exceeds R_est.  So the loaded kernel never has more than R_est registers; a GPU test pins that it
+  // does not spill either.
   {
     const int rest = std::max(24, std::min(L.regs, regs_limit(NT)));
+    std::vector<int> caps;
     std::string primary;
     if (const char* fc = getenv("KF_MAXNREG")) {   // experiments only: force a register cap
       primary = "__maxnreg__(" + std::to_string(atoi(fc)) + ")";
     } else if (L.minblocks >= 0) {
       const int smem_ctas = 233472 / std::max(1, L.smem + 1024);
       const int minb = L.minblocks > 0 ? L.minblocks : std::max(1, std::min({smem_ctas, 2048 / std::max(1, NT), 8}));
-      const int cap = std::max(24, std::min(regs_limit(NT * minb), rest));
-      primary = "__maxnreg__(" + std::to_string(cap) + ")";
+      for (int m = minb; m >= 1; m--) {
+        const int c = std::max(24, std::min(regs_cap(NT, m), rest));
+        if (caps.empty() || c > caps.back()) caps.push_back(c);
+      }
+      primary = "__maxnreg__(KF_CAP)";
     } else {
       primary = "__launch_bounds__(NT)";
     }
-    o << "#define KF_REST " << rest << "\n#ifndef KF_NO_MAXNREG\n#define KF_BOUNDS " << primary
-      << "\n#else\n#define KF_BOUNDS __maxnreg__(KF_REST)\n#endif\n";
+    if (caps.empty() || caps.back() < rest) caps.push_back(rest);
+    o << "#define KF_REST " << rest << "\n// KF_CAPS";
+    for (int c : caps) o << " " << c;
+    o << "\n";
+    if (L.minblocks >= 0 && !getenv("KF_MAXNREG"))
+      o << "#ifndef KF_CAP\n#define KF_CAP " << caps[0] << "\n#endif\n#define KF_BOUNDS __maxnreg__(KF_CAP)\n";
+    else
+      o << "#ifndef KF_CAP\n#define KF_BOUNDS " << primary << "\n#else\n#define KF_BOUNDS __maxnreg__(KF_CAP)\n#endif\n";
   }
   o << "extern \"C\" __global__ void KF_BOUNDS " << cg.name << "(const __grid_constant__ KfArgs a) {\n";
   // pointer arithmetic from the __shared__ array keeps the shared state space (LDS/STS, 32-bit

@@ -151,6 +151,7 @@ int validate_plan_groups(const Program& p, const Plan& pl, const std::vector<kf_
 std::vector<int> quotient_order(const Program& p, const Plan& pl);   // empty if cyclic
 bool regs_ok(const GroupLowering& L, const kf_target& t);              // V8 (Eq. 2, Eq. 3)
 int regs_limit(int threads);                                            // registers per thread of a CTA
+int regs_cap(int threads, int m);                                       // ... with m CTAs per SM resident
 int check_kinship(const Program& p, const std::vector<int>& g, int gi, kf_violation* why);
 int check_convex(const Program& p, const std::vector<int>& g, int gi, kf_violation* why);
 int check_hazard(const Program& p, const std::vector<int>& g, const GroupLowering& L, int gi, kf_violation* why);

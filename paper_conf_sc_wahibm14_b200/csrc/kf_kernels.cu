@@ -159,18 +159,23 @@ __global__ void fill_xy_sectors(FillList L, Geom g, int px, int py, int frozen_o
 }
 
 // Copy every element that is not interior (ghost shell and padding) from src to dst:
-// renamed copies of an array share its frozen ghost values (R9).
+// renamed copies of an array share its frozen ghost values (R9).  One CTA per padded row
+// (grid-stride): ghost rows / planes whole, interior rows only their x ghost + padding ends.
 template <typename T>
 __global__ void copy_shell(T* __restrict__ dst, const T* __restrict__ src, Geom g) {
-  const long long total = (long long)g.plane * (g.nz + 2 * g.gz);
-  for (long long idx = blockIdx.x * (long long)blockDim.x + threadIdx.x; idx < total;
-       idx += (long long)gridDim.x * blockDim.x) {
-    const int zz = int(idx / g.plane);
-    const long long o = idx % g.plane;
-    const int yy = int(o / g.pitch), xx = int(o % g.pitch);
-    const bool interior = zz >= g.gz && zz < g.gz + g.nz && yy >= g.gy && yy < g.gy + g.ny && xx >= g.xoff &&
-                          xx < g.xoff + g.nx;
-    if (!interior) dst[idx] = src[idx];
+  const int rows = (g.ny + 2 * g.gy) * (g.nz + 2 * g.gz);
+  for (int r = blockIdx.x; r < rows; r += gridDim.x) {
+    const int zz = r / (g.ny + 2 * g.gy), yy = r - zz * (g.ny + 2 * g.gy);
+    const long long o = (long long)zz * g.plane + (long long)yy * g.pitch;
+    const bool inner = zz >= g.gz && zz < g.gz + g.nz && yy >= g.gy && yy < g.gy + g.ny;
+    const int skip0 = inner ? g.xoff : int(g.pitch), skip1 = inner ? g.xoff + g.nx : int(g.pitch);
+    for (int x = threadIdx.x; x < int(g.pitch); x += blockDim.x) {
+      if (x >= skip0 && x < skip1) {   // jump over the interior
+        x = skip1 - 1 - (skip1 - 1 - x) % int(blockDim.x);
+        continue;
+      }
+      dst[o + x] = src[o + x];
+    }
   }
 }
 
@@ -264,10 +269,10 @@ cudaError_t launch_fill_xy_multi(void* const* bufs, int n, int px, int py, int e
 }
 
 cudaError_t launch_copy_shell(void* dst, const void* src, int es, const Geom& g, cudaStream_t s) {
-  long long n = (long long)g.plane * (g.nz + 2 * g.gz);
-  int nb = blocks_for(n);
-  if (es == 4) copy_shell<float><<<nb, 256, 0, s>>>((float*)dst, (const float*)src, g);
-  else copy_shell<double><<<nb, 256, 0, s>>>((double*)dst, (const double*)src, g);
+  const long long rows = (long long)(g.ny + 2 * g.gy) * (g.nz + 2 * g.gz);
+  const int nb = int(rows < 148 * 32 ? rows : 148 * 32);
+  if (es == 4) copy_shell<float><<<nb, 128, 0, s>>>((float*)dst, (const float*)src, g);
+  else copy_shell<double><<<nb, 128, 0, s>>>((double*)dst, (const double*)src, g);
   return cudaGetLastError();
 }
 

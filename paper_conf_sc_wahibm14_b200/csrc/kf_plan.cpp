@@ -443,6 +443,13 @@ int regs_limit(int threads) {
   return std::min(255, 16384 / (per_quadrant * 32) / 8 * 8);
 }
 
+// Register cap that keeps m CTAs of NT threads resident per SM: their m*warps warps spread evenly
+// over the 4 sub-partitions (ncu: 3 CTAs of 5 warps at 126 registers fit, 4 warps per quadrant).
+int regs_cap(int threads, int m) {
+  const int warps = std::max(1, m) * ((threads + 31) / 32);
+  return std::min(255, 16384 / (((warps + 3) / 4) * 32) / 8 * 8);
+}
+
 // V8 = Eq. 2 (R_T <= R_Max) and Eq. 3 with one CTA per SM (Thr * R_T <= R_SMX, per sub-partition)
 bool regs_ok(const GroupLowering& L, const kf_target& t) {
   return L.regs <= t.regs_per_thread_max && L.regs <= regs_limit(L.threads);

@@ -85,7 +85,8 @@ struct Compiled {
   std::vector<char> cubin;
   std::string log;
   int regs_ptxas = -1, spill = -1;
-  bool nocap = false;   // compiled with KF_NO_MAXNREG (the fallback build at __maxnreg__(R_est))
+  bool nocap = false;   // a fallback build ("#define KF_CAP c" prepended)
+  int cap_idx = -1;     // position on the source's KF_CAPS ladder (-1: the primary build)
 };
 
 static Compiled nvrtc_compile(const std::string& src, const std::string& name) {
@@ -113,7 +114,7 @@ static Compiled nvrtc_compile(const std::string& src, const std::string& name) {
   nvrtcGetCUBIN(prog, c.cubin.data());
   nvrtcDestroyProgram(&prog);
   if (const char* dir = getenv("KF_DUMP_DIR")) {   // debugging aid: keep the generated source and cubin
-    std::string base = std::string(dir) + "/" + name + (src.rfind("#define KF_NO_MAXNREG", 0) == 0 ? "_nomaxnreg" : "");
+    std::string base = std::string(dir) + "/" + name + (src.rfind("#define KF_CAP", 0) == 0 ? "_cap" + std::to_string(atoi(src.c_str() + 15)) : "");
     if (FILE* f = fopen((base + ".log").c_str(), "w")) { fwrite(c.log.data(), 1, c.log.size(), f); fclose(f); }
     if (FILE* f = fopen((base + ".cu").c_str(), "w")) { fwrite(src.data(), 1, src.size(), f); fclose(f); }
     if (FILE* f = fopen((base + ".cubin").c_str(), "wb")) { fwrite(c.cubin.data(), 1, c.cubin.size(), f); fclose(f); }
@@ -138,6 +139,34 @@ static int source_rest(const std::string& src) {
   return p == std::string::npos ? 255 : atoi(src.c_str() + p + 16);
 }
 
+// fallback register caps of a generated kernel ("// KF_CAPS c0 c1 ... R_est")
+static std::vector<int> source_caps(const std::string& src) {
+  std::vector<int> caps;
+  const auto p = src.find("// KF_CAPS");
+  if (p == std::string::npos) return caps;
+  std::istringstream is(src.substr(p + 10, src.find('\n', p) - p - 10));
+  for (int c; is >> c;) caps.push_back(c);
+  return caps;
+}
+
+static bool needs_next(const Compiled& c, const std::string& src) {
+  return c.spill > 0 || c.regs_ptxas > source_rest(src);
+}
+
+// The build after `c` on the cap ladder (c->cap_idx + 1), or nullptr at the end of it.
+static std::shared_ptr<Compiled> compile_next(const std::string& src, const std::string& name, int cap_idx) {
+  const std::vector<int> caps = source_caps(src);
+  // minblocks >= 0 sources start at caps[0] (KF_CAP default): the first fallback is caps[1]
+  const bool capped_primary = src.find("#define KF_BOUNDS __maxnreg__(KF_CAP)\n") != std::string::npos &&
+                              src.find("#ifndef KF_CAP\n#define KF_CAP") != std::string::npos;
+  const int next = cap_idx + 1 + (cap_idx < 0 && capped_primary ? 1 : 0);
+  if (next >= int(caps.size())) return nullptr;
+  auto c = std::make_shared<Compiled>(nvrtc_compile("#define KF_CAP " + std::to_string(caps[next]) + "\n" + src, name));
+  c->cap_idx = next;
+  c->nocap = true;
+  return c;
+}
+
 static std::shared_ptr<Compiled> compile_cached(const std::string& src, const std::string& name) {
   {
     std::lock_guard<std::mutex> lk(g_cache_mu);
@@ -145,11 +174,11 @@ static std::shared_ptr<Compiled> compile_cached(const std::string& src, const st
     if (it != g_cubin_cache.end()) return it->second;
   }
   auto c = std::make_shared<Compiled>(nvrtc_compile(src, name));
-  // the first build must neither spill nor exceed the register model (V8): else the fallback build
-  // at __maxnreg__(R_est)
-  if ((c->spill > 0 || c->regs_ptxas > source_rest(src)) && src.find("#ifndef KF_NO_MAXNREG") != std::string::npos) {
-    c = std::make_shared<Compiled>(nvrtc_compile("#define KF_NO_MAXNREG 1\n" + src, name));
-    c->nocap = true;
+  // the build must neither spill nor exceed the register model (V8): walk down the cap ladder
+  while (needs_next(*c, src)) {
+    auto n = compile_next(src, name, c->cap_idx);
+    if (!n) break;
+    c = n;
   }
   std::lock_guard<std::mutex> lk(g_cache_mu);
   g_cubin_cache[src] = c;
@@ -157,16 +186,11 @@ static std::shared_ptr<Compiled> compile_cached(const std::string& src, const st
 }
 
 // The ptxas statistics come from the NVRTC log, which is empty when NVRTC serves a program from
-// its own on-disk cache (seen on reused GPU boxes): the spill test above then never fires.  The
-// loader checks the function's local memory instead and comes here for the uncapped build.
-static std::shared_ptr<Compiled> compile_nocap(const std::string& src, const std::string& name) {
-  {
-    std::lock_guard<std::mutex> lk(g_cache_mu);
-    auto it = g_cubin_cache.find(src);
-    if (it != g_cubin_cache.end() && it->second->nocap) return it->second;
-  }
-  auto c = std::make_shared<Compiled>(nvrtc_compile("#define KF_NO_MAXNREG 1\n" + src, name));
-  c->nocap = true;
+// its own on-disk cache (seen on reused GPU boxes): the checks above then never fire.  The loader
+// checks the loaded function's registers and local memory instead and comes here for the next cap.
+static std::shared_ptr<Compiled> compile_after(const std::string& src, const std::string& name, int cap_idx) {
+  auto c = compile_next(src, name, cap_idx);
+  if (!c) return nullptr;
   std::lock_guard<std::mutex> lk(g_cache_mu);
   g_cubin_cache[src] = c;
   return c;
@@ -441,7 +465,7 @@ static void ensure_device(kf_exec* E) {
   E->device = dev;
   const Program& p = E->prog->p;
   for (auto& g : E->G) {
-    for (int attempt = 0; attempt < 2; attempt++) {
+    for (int attempt = 0; attempt < 12; attempt++) {
       ckd(drv().moduleLoadData(&g.mod, g.comp->cubin.data()), ("cuModuleLoadData " + g.cg.name).c_str());
       ckd(drv().moduleGetFunction(&g.fn, g.mod, g.cg.name.c_str()), "cuModuleGetFunction");
       ckd(drv().funcSetAttribute(g.fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, g.smem),
@@ -449,10 +473,10 @@ static void ensure_device(kf_exec* E) {
       drv().funcGetAttribute(&g.regs, CU_FUNC_ATTRIBUTE_NUM_REGS, g.fn);
       drv().funcGetAttribute(&g.local, CU_FUNC_ATTRIBUTE_LOCAL_SIZE_BYTES, g.fn);
       drv().funcGetAttribute(&g.maxthr, CU_FUNC_ATTRIBUTE_MAX_THREADS_PER_BLOCK, g.fn);
-      // the register cap must not cost local memory (spills): rebuild without it
-      if ((g.local > 0 || g.regs > source_rest(g.cg.source)) && !g.comp->nocap &&
-          g.cg.source.find("#ifndef KF_NO_MAXNREG") != std::string::npos) {
-        g.comp = compile_nocap(g.cg.source, g.cg.name);
+      // no spills, no more registers than R_est: else the next build of the cap ladder
+      std::shared_ptr<Compiled> nx;
+      if ((g.local > 0 || g.regs > source_rest(g.cg.source)) && (nx = compile_after(g.cg.source, g.cg.name, g.comp->cap_idx))) {
+        g.comp = nx;
         if (drv().moduleUnload) drv().moduleUnload(g.mod);
         g.mod = nullptr;
         g.fn = nullptr;

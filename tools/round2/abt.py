@@ -48,7 +48,16 @@ def main():
                 os.environ[k] = o
         sb = ex.scratch_bytes()
         scr = torch.empty(sb, dtype=torch.uint8, device="cuda") if sb else None
-        runs.append((v, ex, scr, [], []))
+        if v.get("dist"):   # loopback kf_dist over one part: periodic fills overlapped with interior tiles
+            d = kf.Dist([ex], 1, 1)
+            d.set_overlap(True)
+            runner = type("R", (), {})()
+            runner.ex = ex
+            runner.run = (lambda d_: (lambda dev_, scr_, n: d_.run([dev_], [scr_], n)))(d)
+            runner.d = d
+        else:
+            runner = ex
+        runs.append((v, runner, scr, [], []))
     for _ in range(spec.get("rounds", 5)):
         for v, ex, scr, st, gt_ in runs:
             ex.run(dev, scr, 2)
@@ -59,14 +68,16 @@ def main():
             e1.record()
             torch.cuda.synchronize()
             st.append(e0.elapsed_time(e1) / steps)
-            ex.set_profiling(True)
+            ex.ex.set_profiling(True) if hasattr(ex, "d") else ex.set_profiling(True)
             ex.run(dev, scr, steps)
             torch.cuda.synchronize()
-            gms, _ = ex.group_times()
-            ex.set_profiling(False)
+            e_ = ex.ex if hasattr(ex, "d") else ex
+            gms, _ = e_.group_times()
+            e_.set_profiling(False)
             gt_.append([g / steps for g in gms])
     for v, ex, scr, st, gt_ in runs:
         med = [statistics.median(x) for x in zip(*gt_)]
+        ex = ex.ex if hasattr(ex, "d") else ex
         gi = [ex.group_info(g) for g in range(ex.info().n_groups)]
         print(json.dumps({"variant": v.get("name", v), "ms_per_step": round(statistics.median(st), 4),
                           "ms_all": [round(x, 4) for x in st], "fills_per_step": ex.info().fills_per_step,
