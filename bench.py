@@ -625,7 +625,25 @@ def run_kf(args):
         tkw["internal_axes"] = (1 if px > 1 else 0) | (2 if py > 1 else 0)
     target = kf.Target(**tkw)
     prog = kf.Program(desc)          # the per-GPU sub-domain program
-    plan, plan_kind = (None, None) if args.plan == "select" else choose_plan(prog, target, args.plan)
+    committed = None
+    if args.plan == "auto":
+        # the committed configuration of config 3: plan and per-group launch configurations chosen by
+        # measured selection + per-group autotuning on B200 in an earlier run (source recorded in the
+        # file), replayed as is -- reproducible, and the ncu evidence under profiles/ names its kernels
+        path = os.path.join(ROOT, "profiles", "bench_timed_config.json")
+        if (args.workload == "weather" and S == 1 and not args.relax_all and not args.tuned and world == 1
+                and not args.ghostwrite and os.path.exists(path)):
+            committed = json.load(open(path))
+            if committed.get("ghostwrite", 0) != tkw["ghostwrite"]:
+                committed = None
+        if committed is None:
+            args.plan = "select"
+    if committed is not None:
+        plan = committed["plan_labels"]
+        plan_kind = f"committed tuned configuration (profiles/bench_timed_config.json; {committed.get('source', '')})"
+        args.tuned = json.dumps(committed["per_group_launch_config"])
+    else:
+        plan, plan_kind = (None, None) if args.plan == "select" else choose_plan(prog, target, args.plan)
 
     def new_dist_info():
         """A fresh NCCL unique id (broadcast from rank 0) for every communicator kf.Dist creates."""
@@ -918,9 +936,10 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="kf", choices=["kf", "reference"])
     ap.add_argument("--workload", default="weather")
-    ap.add_argument("--plan", default="select",
-                    help="select: measured choice among the searches' candidates; best: HGGA/brute on projected "
-                         "time; unfused; hand; or a JSON label list (config.plan_labels of an earlier run)")
+    ap.add_argument("--plan", default="auto",
+                    help="auto: config 3 replays the committed tuned configuration (profiles/bench_timed_config.json), "
+                         "other workloads select; select: measured choice among the searches' candidates + autotune; "
+                         "best: HGGA/brute on projected time; unfused; hand; or a JSON label list")
     ap.add_argument("--relax-all", type=int, default=0, help="weather: rename every written array (KF_PROG_RELAX_ALL)")
     ap.add_argument("--unroll", type=int, default=1, help="NEXT-4 temporal fusion: plan over S timesteps as one step")
     ap.add_argument("--tile", default=None)
