@@ -598,7 +598,7 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
           if (ring >= 0 && need_sts.count(v)) {
             const Ring& R = L.rings[ring];
             o << "      if (ce" << k << rs << ") P" << ring << "_" << slot(ring, -L.delay.at(k) + uu) << "[cb" << R.px << rs << " - "
-              << (oy * R.px + ox) << "] = " << vals[si] << ";\n";
+              << (oy * R.px + (clo[0] - R.ax_lo)) << "] = " << vals[si] << ";\n";
           }
           if (out_index(v) >= 0) any_out = true;
         }
@@ -855,9 +855,10 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
           const int ring = L.ring_of(v);
           if (ring >= 0 && need_sts.count(v)) {
             const Ring& R = L.rings[ring];
+            const int oxr = clo[0] - R.ax_lo;   // ring column of canvas x 0 is -oxr
             const std::string base = "P" + std::to_string(ring) + "_" + std::to_string(slot(ring, -L.delay.at(k))) + "[cb" +
-                                     std::to_string(R.px) + "_r0 - " + std::to_string(oy * R.px + ox);
-            if (mod2(PSH + ox) == 0)   // the pair is aligned in this ring
+                                     std::to_string(R.px) + "_r0 - " + std::to_string(oy * R.px + oxr);
+            if (mod2(PSH + oxr) == 0)   // the pair is aligned in this ring
               o << "      if (" << c0 << " && " << c1 << ") *(real2*)&" << base << "] = real2{" << v0[si] << ", " << v1[si]
                 << "};\n      else { if (" << c0 << ") " << base << "] = " << v0[si] << "; if (" << c1 << ") " << base
                 << " + 1] = " << v1[si] << "; }\n";
@@ -1051,7 +1052,9 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
         const Ring& R = L.rings[oi.ring];
         for (int uu = 0; uu < U; uu++) {
           const int om = ((-L.delay.at(k) + uu) % R.slots + R.slots) % R.slots;
-          o << "        real* w" << oi.ring << "_" << uu << " = P" << oi.ring << "_" << om << ";\n";
+          // writes use the producer's region coordinates; the ring box starts ax_lo - blo0 columns
+          // further left (16-byte aligned box origin)
+          o << "        real* w" << oi.ring << "_" << uu << " = P" << oi.ring << "_" << om << " + " << (R.ax_lo - R.blo[0]) << ";\n";
         }
       }
     o << "        const int gx0 = x0 - " << e.elo[0] << ", gy0 = y0 - " << e.elo[1] << ";\n";

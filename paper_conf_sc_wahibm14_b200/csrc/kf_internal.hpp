@@ -127,6 +127,7 @@ struct GroupLowering {
   std::set<Ver> live_out_set;
   std::vector<Ring> rings;
   int smem = 0, regs = 0, depth = 0;
+  int thrld = 0, pts = 1;                 // register model inputs (V8): values held, points per thread
   int mbar_off = 0;
   int tile[3];
   int stages = 2, threads = 256, zunroll = 1;

@@ -147,12 +147,21 @@ GroupLowering lower_group(const Program& p, const std::vector<int>& g, const kf_
   const int es = p.es, TX = t.tile[0], TY = t.tile[1], S = t.stages, U = t.zunroll;
   auto finish_ring = [&](Ring& r) {
     const int a = 16 / es;
-    // TMA box x start must be 16-byte aligned: round the lower x extent of a live-in box up to a
-    // multiple of 16/es elements (ceil toward +inf also for negative extents).
-    r.ax_lo = r.live_in ? (r.blo[0] >= 0 ? (r.blo[0] + a - 1) / a * a : -((-r.blo[0]) / a * a)) : r.blo[0];
+    // Box x start 16-byte aligned: the lower x extent rounded up to a multiple of 16/es elements
+    // (ceil toward +inf also for negative extents).  Live-in boxes need it for TMA (R20a); in-group
+    // rings (round 2) so every ring row shares the canvas' pair / 16-byte alignment: pair stores are
+    // single 16-byte stores and pair loads never split (ncu: split STS.64 / LDS.64 were half of the
+    // excess shared wavefronts of the flux groups).
+    static const bool legacy = getenv("KF_RING_LEGACY") != nullptr;   // A/B only: the round-1 layout
+    r.ax_lo = r.blo[0] >= 0 ? (r.blo[0] + a - 1) / a * a : -((-r.blo[0]) / a * a);
+    if (legacy && !r.live_in) r.ax_lo = r.blo[0];
     r.wx = TX + r.ax_lo + r.bhi[0];
     r.hy = TY + r.blo[1] + r.bhi[1];
-    r.px = int(rup(r.wx, 16 / es));
+    // row pitch: a multiple of 16 bytes and an ODD number of 16-byte units, so the rows a column of
+    // threads reads (halo columns: consecutive lanes on consecutive rows) fall on distinct bank groups
+    // (ncu round 2: an even pitch made them 2-way conflicts)
+    r.px = int(rup(r.wx, a));
+    if ((r.px / a) % 2 == 0 && !legacy) r.px += a;
     r.plane_bytes = int(rup(int64_t(r.px) * r.hy * es, 128));
   };
   // ---- live-in rings (TMA staged)
@@ -299,6 +308,8 @@ GroupLowering lower_group(const Program& p, const std::vector<int>& g, const kf_
     }
     const int thrld = canvas ? int(all.size()) : kmax;
     L.regs = 32 * U + (es / 4) * P * (thrld + depth);
+    L.thrld = thrld;
+    L.pts = P;
   }
   return L;
 }
@@ -503,10 +514,19 @@ uint64_t group_bytes(const Program& p, const std::vector<int>& g, uint64_t* rd, 
 }
 
 double model_time(const Program& p, const GroupLowering& L, const kf_target& t, uint64_t bytes) {
-  // Calibrated on B200 (profiles/round1_summary.md): ~17 issue slots of fixed cost per point of
-  // an extended region plus ~1.5 per RPN node / store; ~2.5e13 thread-instructions/s sustained;
-  // compulsory bytes at 79% of nominal HBM (the measured copy rate); memory and issue overlap
-  // by half the shorter of the two.  A model, not a measurement (reported beside measured times).
+  // NEXT-2 (R22, recalibrated in round 2 on 129 measured groups: 8 candidate plans' groups under the
+  // default launch configuration + the autotuned configurations of the bench plan, clamped canvas
+  // loads; median error 5 %, max 24 %, tools/round2/model_fit.py, profiles/round2_summary.md).
+  // The paper's Eq. 9 idea -- the memory bound scaled by the effectiveness of blocking B_eff
+  // -- with B_eff from the warps a SM keeps resident:
+  //   CTAs/SM   = the shared-memory / thread limit, lowered while a register NEED estimate
+  //               (R_adr*U + 0.6*(es/4)*P*(ThrLD + depth): the register model with RegFac 0.6, the
+  //               reuse ptxas achieves) does not fit the per-sub-partition register file (Eq. 3)
+  //   warps     = CTAs * warps/CTA (a pair-canvas thread counts twice: two independent points)
+  //   t_mem     = bytes / (copy rate 0.8185 * nominal) / 0.98 / min(1, warps / 8)
+  //   t_smem    = canvas shared-memory traffic / (128 B/clk * n_sm * 1.9 GHz) / 0.7
+  //   t         = max(t_mem, t_smem) + 0.1 * t_issue / min(1, warps / 24)   (x0.5 for pairs)
+  // t_issue: ~17 issue slots of fixed cost per point of an extended region plus ~1.5 per RPN node.
   const double T = double(L.tile[0]) * L.tile[1];
   double work = 0.0;
   for (int k : L.kernels) {
@@ -517,22 +537,24 @@ double model_time(const Program& p, const GroupLowering& L, const kf_target& t, 
     for (auto& st : p.kernels[k].stmts) ops += int(st.rpn.size()) + 1;
     work += (R / T) * (17.0 + 1.5 * ops);
   }
-  // issue efficiency falls with the warps an SM can hold (SMEM-limited CTAs x warps per CTA):
-  // full rate from 32 resident warps, proportionally less below (latency no longer hidden)
-  const int ctas = std::max(1, std::min(2048 / std::max(32, L.threads), 233472 / std::max(1, L.smem + 1024)));
-  const double warps = std::min(64.0, double(ctas) * (L.threads / 32));
-  const double eff = std::min(1.0, warps / 32.0);
-  const double t_comp = double(p.npts) * work / (2.5e13 * eff);
-  const double t_mem = double(bytes) / (0.79 * t.hbm_bytes_per_s);
-  // shared-memory bandwidth (the canvas plan's loads, ring stores and TMA writes per tile plane) at
-  // 128 B/clk/SM on n_sm SMs at 1.9 GHz
+  const int old_ctas = std::max(1, std::min(2048 / std::max(32, L.threads), 233472 / std::max(1, L.smem + 1024)));
+  const double old_eff = std::min(1.0, std::min(64.0, double(old_ctas) * (L.threads / 32)) / 32.0);
+  const double t_comp = double(p.npts) * work / (2.5e13 * old_eff);
   const CanvasPlan cv = plan_canvas(p, L);
   const double per_plane = (cv.lds_bytes + cv.sts_bytes + cv.tma_bytes) / std::max(1, L.zunroll);
   const double t_smem = double(p.npts) / T * per_plane / (128.0 * t.n_sm * 1.9e9);
+  // resident warps
+  const int need = int(32 * L.zunroll + 0.6 * (p.es / 4) * L.pts * (L.thrld + L.depth));
+  int ctas = std::max(1, std::min({233472 / std::max(1, L.smem + 1024), 2048 / std::max(32, L.threads), 32}));
+  while (ctas > 1 && regs_cap(L.threads, ctas) < need) ctas--;
+  const bool pair = cv.ok && cv.pair;
+  const double warps = double(ctas) * ((L.threads + 31) / 32) * (pair ? 2.0 : 1.0);
+  const double t_mem = double(bytes) / (0.8185 * t.hbm_bytes_per_s) / 0.98 / std::min(1.0, warps / 8.0);
+  const double t_issue = 0.1 * t_comp / std::min(1.0, warps / 24.0) * (pair ? 0.5 : 1.0);
   if (getenv("KF_DEBUG_MODEL"))
-    fprintf(stderr, "model: group of %zu kernels: mem %.3f ms, smem %.3f ms (lds %.0f sts %.0f tma %.0f B/plane, canvas %d), comp %.3f ms\n",
-            L.kernels.size(), t_mem * 1e3, t_smem * 1e3, cv.lds_bytes, cv.sts_bytes, cv.tma_bytes, int(cv.ok), t_comp * 1e3);
-  return t_mem + t_comp - 0.5 * std::min(t_mem, t_comp) + 5e-6;
+    fprintf(stderr, "model: group of %zu kernels: mem %.3f ms, smem %.3f ms (lds %.0f sts %.0f tma %.0f B/plane, canvas %d), comp %.3f ms, ctas %d warps %.0f\n",
+            L.kernels.size(), t_mem * 1e3, t_smem * 1e3, cv.lds_bytes, cv.sts_bytes, cv.tma_bytes, int(cv.ok), t_comp * 1e3, ctas, warps);
+  return std::max(t_mem, t_smem / 0.7) + t_issue + 5e-6;
 }
 
 void check_target(const kf_target* t) {
