@@ -234,8 +234,6 @@ def schedule(prog: Program, grp: List[int], target: Target):
     smem = 0
     for r in res:
         px = _roundup(r[3], 16 // es)
-        if (px // (16 // es)) % 2 == 0:   # an odd number of 16-byte units per row (bank groups)
-            px += 16 // es
         plane = _roundup(px * r[4] * es, 128)
         smem += r[5] * plane
     smem += 8 * S + 128

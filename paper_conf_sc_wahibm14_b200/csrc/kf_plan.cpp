@@ -152,16 +152,15 @@ GroupLowering lower_group(const Program& p, const std::vector<int>& g, const kf_
     // rings (round 2) so every ring row shares the canvas' pair / 16-byte alignment: pair stores are
     // single 16-byte stores and pair loads never split (ncu: split STS.64 / LDS.64 were half of the
     // excess shared wavefronts of the flux groups).
-    static const bool legacy = getenv("KF_RING_LEGACY") != nullptr;   // A/B only: the round-1 layout
+    const bool legacy = getenv("KF_RING_LEGACY") != nullptr;   // A/B only: round-1 in-group ring origins
     r.ax_lo = r.blo[0] >= 0 ? (r.blo[0] + a - 1) / a * a : -((-r.blo[0]) / a * a);
     if (legacy && !r.live_in) r.ax_lo = r.blo[0];
     r.wx = TX + r.ax_lo + r.bhi[0];
     r.hy = TY + r.blo[1] + r.bhi[1];
-    // row pitch: a multiple of 16 bytes and an ODD number of 16-byte units, so the rows a column of
-    // threads reads (halo columns: consecutive lanes on consecutive rows) fall on distinct bank groups
-    // (ncu round 2: an even pitch made them 2-way conflicts)
+    // row pitch: a multiple of 16 bytes.  (An odd number of 16-byte units would remove the 2-way
+    // bank conflicts of the halo-column threads, but its ~5 % more shared memory cost the flux groups
+    // a CTA per SM: measured 3.07 vs 2.58 ms per step, round 2 -- not used.)
     r.px = int(rup(r.wx, a));
-    if ((r.px / a) % 2 == 0 && !legacy) r.px += a;
     r.plane_bytes = int(rup(int64_t(r.px) * r.hy * es, 128));
   };
   // ---- live-in rings (TMA staged)
