@@ -225,10 +225,7 @@ def schedule(prog: Program, grp: List[int], target: Target):
                 continue
             span = max(D[c] - d[2] for c, offs in rd for d in offs) - D[p] + 1 + (target.zunroll - 1)
             (lo, hi) = ext[p]
-            # box x start 16-byte aligned as for live-ins (round 2: pair / 16-byte alignment of every ring)
-            al = 16 // es
-            lox = -((-lo[0]) // al) * al
-            res.append(("mid", x, v, TX + lox + hi[0], TY + lo[1] + hi[1], span, 0, 0))
+            res.append(("mid", x, v, TX + lo[0] + hi[0], TY + lo[1] + hi[1], span, 0, 0))
     if target.ringunroll:   # ring depths rounded up to powers of two (stream loop unrolled, R20b)
         res = [r[:5] + (1 << (r[5] - 1).bit_length(),) + r[6:] for r in res]
     smem = 0

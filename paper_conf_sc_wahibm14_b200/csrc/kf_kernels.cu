@@ -286,14 +286,34 @@ cudaError_t launch_copy_box(void* dst, long long dpitch, long long dplane, const
   return cudaGetLastError();
 }
 
+// A box whose rows are whole 16-byte units at 16-byte aligned addresses (ghost-deep x strips of
+// fp64 with an even ghost width, whole padded rows of y strips) is copied as uint4 elements.
+static bool vec16(const BoxCopy& b, int es) {
+  const long long m = 16;
+  return (reinterpret_cast<uintptr_t>(b.dst) % m) == 0 && (reinterpret_cast<uintptr_t>(b.src) % m) == 0 &&
+         (b.w * (long long)es) % m == 0 && (b.dpitch * es) % m == 0 && (b.spitch * es) % m == 0 &&
+         (b.dplane * es) % m == 0 && (b.splane * es) % m == 0;
+}
+
 cudaError_t launch_copy_boxes(const BoxCopy* boxes, int n, int es, cudaStream_t s) {
+  bool all16 = true;
+  for (int i = 0; i < n; i++) all16 = all16 && vec16(boxes[i], es);
+  const int f = all16 ? 16 / es : 1;   // elements per copied unit
   for (int b0 = 0; b0 < n; b0 += kMaxBoxes) {
     const int m = n - b0 < kMaxBoxes ? n - b0 : kMaxBoxes;
     BoxList L{};
     long long most = 0;
     for (int i = 0; i < m; i++) {
-      L.box[i] = boxes[b0 + i];
-      const long long e = (long long)L.box[i].w * L.box[i].h * L.box[i].d;
+      BoxCopy b = boxes[b0 + i];
+      if (f > 1) {   // geometry in 16-byte units
+        b.w /= f;
+        b.dpitch /= f;
+        b.spitch /= f;
+        b.dplane /= f;
+        b.splane /= f;
+      }
+      L.box[i] = b;
+      const long long e = (long long)b.w * b.h * b.d;
       if (e >= (1LL << 32)) return cudaErrorInvalidValue;
       most = e > most ? e : most;
     }
@@ -301,7 +321,8 @@ cudaError_t launch_copy_boxes(const BoxCopy* boxes, int n, int es, cudaStream_t 
     const long long nb = (most + 255) / 256;
     const long long cap = (148LL * 8 + m - 1) / m;   // ~8 CTAs per SM over all boxes
     dim3 grid(unsigned(nb < cap ? nb : cap), unsigned(m));
-    if (es == 4) copy_boxes<float><<<grid, 256, 0, s>>>(L);
+    if (f > 1) copy_boxes<uint4><<<grid, 256, 0, s>>>(L);
+    else if (es == 4) copy_boxes<float><<<grid, 256, 0, s>>>(L);
     else copy_boxes<double><<<grid, 256, 0, s>>>(L);
   }
   return cudaGetLastError();

@@ -147,14 +147,11 @@ GroupLowering lower_group(const Program& p, const std::vector<int>& g, const kf_
   const int es = p.es, TX = t.tile[0], TY = t.tile[1], S = t.stages, U = t.zunroll;
   auto finish_ring = [&](Ring& r) {
     const int a = 16 / es;
-    // Box x start 16-byte aligned: the lower x extent rounded up to a multiple of 16/es elements
-    // (ceil toward +inf also for negative extents).  Live-in boxes need it for TMA (R20a); in-group
-    // rings (round 2) so every ring row shares the canvas' pair / 16-byte alignment: pair stores are
-    // single 16-byte stores and pair loads never split (ncu: split STS.64 / LDS.64 were half of the
-    // excess shared wavefronts of the flux groups).
-    const bool legacy = getenv("KF_RING_LEGACY") != nullptr;   // A/B only: round-1 in-group ring origins
-    r.ax_lo = r.blo[0] >= 0 ? (r.blo[0] + a - 1) / a * a : -((-r.blo[0]) / a * a);
-    if (legacy && !r.live_in) r.ax_lo = r.blo[0];
+    // TMA box x start must be 16-byte aligned: round the lower x extent of a live-in box up to a
+    // multiple of 16/es elements (ceil toward +inf also for negative extents).  (Round 2 tried the
+    // same for in-group rings, so pair stores never split: no gain measured, KF_RING_ALIGN=1.)
+    const bool align = r.live_in || getenv("KF_RING_ALIGN") != nullptr;
+    r.ax_lo = !align ? r.blo[0] : r.blo[0] >= 0 ? (r.blo[0] + a - 1) / a * a : -((-r.blo[0]) / a * a);
     r.wx = TX + r.ax_lo + r.bhi[0];
     r.hy = TY + r.blo[1] + r.bhi[1];
     // row pitch: a multiple of 16 bytes.  (An odd number of 16-byte units would remove the 2-way

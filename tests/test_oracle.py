@@ -465,16 +465,16 @@ def test_bytes_closed_form_and_monotone(seed):
 
 def test_resource_model_worked_example():
     """V7 model (R20), hand-worked for tiny {K1,K2}, fp32, tile 32x16, S=2 stages, U=2 planes/iteration:
-    delays D(K1)=0, D(K2)=1 (K2 reads v at dz=+1).  Row pitch: a multiple of 16 bytes (4 fp32).
-    u (live-in): box x extent below T 2 -> 4 (16-byte box start, R20a), width 32+4+2=38 -> row 40,
+    delays D(K1)=0, D(K2)=1 (K2 reads v at dz=+1).
+    u (live-in): box x extent below T 2 -> 4 (16-byte TMA start, R20a), width 32+4+2=38 -> row 40,
       height 20, A=1-0=1, B=-1-0=-1 -> span 3, slots 3+U*S-1=6, plane roundup(40*20*4,128)=3200
-    v (in-group): x extent below T 1 -> 4 (16-byte box start, round 2), width 32+4+1=37 -> row 40,
-      height 18, span (1-(-1))-0+1 = 3, slots 3+(U-1)=4, plane roundup(40*18*4,128)=2944
-    total = 6*3200 + 4*2944 + 8*2 + 128 = 31120;  with U=1: 4*3200 + 3*2944 + 144 = 21776."""
+    v (in-group): box 34x18 -> row 36, span (1-(-1))-0+1 = 3, slots 3+(U-1)=4,
+      plane roundup(36*18*4,128)=2688
+    total = 6*3200 + 4*2688 + 8*2 + 128 = 30096;  with U=1: 4*3200 + 3*2688 + 144 = 21008."""
     s = L.schedule(P.tiny(), [0, 1], L.Target(tile=(32, 16, 0), zunroll=2))
     assert s["delay"] == {0: 0, 1: 1}
-    assert s["smem"] == 6 * 3200 + 4 * 2944 + 16 + 128 == 31120
-    assert L.schedule(P.tiny(), [0, 1], L.Target(tile=(32, 16, 0), zunroll=1))["smem"] == 21776
+    assert s["smem"] == 6 * 3200 + 4 * 2688 + 16 + 128 == 30096
+    assert L.schedule(P.tiny(), [0, 1], L.Target(tile=(32, 16, 0), zunroll=1))["smem"] == 21008
 
 
 def test_L25_radius4_stencil_closed_form_through_stress_program():

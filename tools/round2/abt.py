@@ -31,7 +31,8 @@ def main():
     steps = spec.get("steps", 10)
     runs = []
     for v in spec["variants"]:
-        tuned = [list(c) for c in spec["tuned"]]
+        plan = v.get("plan", spec["plan"])
+        tuned = [list(c) for c in v.get("tuned", spec["tuned"])]
         for g, c in v.get("override", {}).items():
             tuned[int(g)] = c
         old = {}
