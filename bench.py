@@ -696,6 +696,10 @@ def run_kf(args):
     clocks = clk.summary()
     # per-group device times over a second timed region (events on the launch stream)
     ms_prof, (gms, nlaunch) = time_runner(rn, dev, args.steps, 1, stream, profile=True)
+    # sustained rate: a longer region (the flux groups slow down once the board reaches its power limit)
+    sus_steps = max(200, args.steps)
+    ms_sus, _ = time_runner(rn, dev, sus_steps, 1, stream)
+    ms_sus = max_over_ranks(ms_sus)
     # unfused plan on the same inputs: speedup vs unfused, and the original per-kernel times
     unf = None
     k_ms = None
@@ -817,6 +821,8 @@ def run_kf(args):
         "fills_per_step": info.fills_per_step,
         "projected_ms_per_step": t_proj * 1e3,
         "model_ms_per_step": sum(g.t_model_s for g in per) * 1e3,
+        "sustained": {"steps": sus_steps, "ms_per_step": ms_sus / sus_steps / S,
+                      "value": wl.global_npts * sus_steps * S / (ms_sus / 1e3)},
         "per_group": per_groups,
         "model_error_max": max(mod_err) if mod_err else None,
         "roofline": roofline,
