@@ -430,7 +430,10 @@ AUTOTUNE_CANDIDATES = [  # (tile, stages, zunroll, ringunroll, minblocks, canvas
     # (wave quantisation; measured -2..-4 % on the flux groups)
     ((32, 8, 43), 2, 1, 0, -1, 1, 2, 1), ((32, 8, 43), 2, 1, 0, -1, 1, 2, 0), ((32, 8, 43), 2, 1, 0, -1, 1),
     # taller / wider pair tiles: less halo per point (36x20/512 = 1.41 vs 36x12/256 = 1.69 box/tile)
-    ((32, 16, 43), 2, 1, 0, -1, 1, 2, 1), ((32, 16, 43), 2, 1, 0, -1, 1, 2, 0), ((64, 8, 43), 2, 1, 0, -1, 1, 2, 1)]
+    ((32, 16, 43), 2, 1, 0, -1, 1, 2, 1), ((32, 16, 43), 2, 1, 0, -1, 1, 2, 0), ((64, 8, 43), 2, 1, 0, -1, 1, 2, 1),
+    # three TMA stages for pairs: ncu showed 12 % of the flux group's warp samples waiting on the
+    # mbarrier of the current plane (one plane of prefetch is not enough latency cover)
+    ((32, 8, 43), 3, 1, 0, -1, 1, 2, 1), ((32, 8, 43), 3, 1, 0, -1, 1, 2, 0), ((32, 8, 64), 3, 1, 0, -1, 1, 2, 1)]
 
 
 def cand_kw(base_kw, c):

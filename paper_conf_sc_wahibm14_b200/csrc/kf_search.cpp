@@ -42,9 +42,9 @@ class Evaluator {
         v.ok = false;
       else {
         v.t_model = model_time(p_, L, t_, v.bytes);
-        // the bench autotunes every group's launch configuration; the flux-type groups mostly run
-        // fastest as the pair canvas, so a group is projected at the better of the two (round 2)
-        if (t_.pblock[0] == 1 && t_.pblock[1] == 1 && t_.zunroll == 1 && !getenv("KF_MODEL_POINTS_ONLY")) {
+        // experiment (KF_MODEL_PAIRS): project a group at the better of the point and pair canvas, as
+        // autotuning picks -- its plans measured slower once tuned (round 2), so off by default
+        if (t_.pblock[0] == 1 && t_.pblock[1] == 1 && t_.zunroll == 1 && getenv("KF_MODEL_PAIRS")) {
           kf_target tp = t_;
           tp.pblock[0] = 2;
           tp.pair_zq = 1;
