@@ -768,6 +768,16 @@ def run_kf(args):
                 "share_of_step": gms[g_dom] / max(1e-9, sum(gms)),
                 "algorithmic_bytes_per_launch": gi.bytes_per_launch,
                 "per_group_ms_per_step": [g / args.steps for g in gms]}
+    # on-chip roofline of the same kernel: its canvas shared-memory traffic (loads + stores + TMA
+    # writes per fast iteration, from the lowering) over the SMEM bandwidth (128 B/clk/SM at the
+    # measured SM clock) -- the bound of groups whose halo recompute outweighs their HBM bytes
+    sm_clk = (clocks.get("sm_mhz") or 1965) * 1e6
+    onchip = {"bound": "smem", "achieved": gi.onchip_bytes_per_launch / (t_launch_ms / 1e3) / 1e9,
+              "peak": 128 * 148 * sm_clk / 1e9, "unit": "GB/s",
+              "algorithmic_bytes_per_launch": gi.onchip_bytes_per_launch,
+              "peak_source": "128 B/clk/SM x 148 SMs x SM clock (B300_MICROARCH / B200_PROFILING)"}
+    onchip["frac"] = onchip["achieved"] / onchip["peak"]
+    roofline["onchip"] = onchip
     achieved_step = bytes_step / (ms / args.steps / 1e3) / 1e9
     # NEXT-2 (Figs. 6-8 analogue): per group measured vs projected vs the original kernels' sum
     per_groups = []

@@ -323,10 +323,13 @@ typedef struct {
 kf_status kf_exec_get_info(const kf_exec* ex, kf_exec_info* out);
 /* Per-group launch details: grid, threads, dynamic SMEM, registers (cuFuncGetAttribute),
  * local (spill) bytes, the loaded function's maximum threads per CTA (-1 before loading),
- * compulsory bytes per launch, kernel name.  name: >= 64 chars. */
+ * compulsory HBM bytes per launch, shared-memory bytes per launch of the canvas fast iterations
+ * (loads + stores + TMA writes; the on-chip roofline's algorithmic bytes), kernel name.
+ * name: >= 64 chars. */
 typedef struct {
   int32_t group, grid, threads, smem_bytes, regs, local_bytes, n_kernels, max_threads;
   uint64_t bytes_per_launch;
+  uint64_t onchip_bytes_per_launch;
   char name[64];
 } kf_group_info;
 kf_status kf_exec_group_info(const kf_exec* ex, int32_t group, kf_group_info* out);

@@ -92,7 +92,7 @@ class kf_exec_info(C.Structure):
 class kf_group_info(C.Structure):
     _fields_ = [("group", C.c_int32), ("grid", C.c_int32), ("threads", C.c_int32), ("smem_bytes", C.c_int32),
                 ("regs", C.c_int32), ("local_bytes", C.c_int32), ("n_kernels", C.c_int32), ("max_threads", C.c_int32),
-                ("bytes_per_launch", C.c_uint64), ("name", C.c_char * 64)]
+                ("bytes_per_launch", C.c_uint64), ("onchip_bytes_per_launch", C.c_uint64), ("name", C.c_char * 64)]
 
 
 class kf_box(C.Structure):

@@ -853,6 +853,12 @@ kf_status kf_exec_group_info(const kf_exec* ex, int32_t group, kf_group_info* ou
     r.n_kernels = int(g.L.kernels.size());
     r.max_threads = g.maxthr;
     r.bytes_per_launch = g.bytes;
+    {
+      const Program& p = ex->prog->p;
+      const CanvasPlan cv = plan_canvas(p, g.L);
+      const double per_plane = (cv.lds_bytes + cv.sts_bytes + cv.tma_bytes) / std::max(1, g.L.zunroll);
+      r.onchip_bytes_per_launch = uint64_t(double(p.npts) / (double(g.L.tile[0]) * g.L.tile[1]) * per_plane);
+    }
     std::strncpy(r.name, g.cg.name.c_str(), sizeof(r.name) - 1);
     *out = r;
   });
