@@ -1,7 +1,7 @@
 """Summarise an ncu --set full report (raw page) into the table used in profiles/*.md."""
 import csv, io, subprocess, sys
 
-M = [("gpu__time_duration.sum", "dur us", 1e-3), ("dram__bytes_read.sum", "dram rd GB", None),
+M = [("gpu__time_duration.sum", "dur us", "time"), ("dram__bytes_read.sum", "dram rd GB", None),
      ("dram__bytes_write.sum", "dram wr GB", None), ("gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed", "dram %", 1),
      ("l1tex__data_pipe_lsu_wavefronts_mem_shared.sum.pct_of_peak_sustained_elapsed", "smem wf %", 1),
      ("l1tex__data_pipe_lsu_wavefronts_mem_shared_op_ld.sum", "ld wf M", 1e-6),
@@ -31,8 +31,10 @@ def main(path):
         vals = []
         for r in data:
             v = float(r[ix[key]].replace(",", "")) if r[ix[key]] else float("nan")
-            if sc is None:
-                v = v if units[ix[key]].lower().startswith("g") else v / 1e9
+            if sc == "time":   # to microseconds whatever unit ncu chose
+                v *= {"nsecond": 1e-3, "ns": 1e-3, "usecond": 1.0, "us": 1.0, "msecond": 1e3, "ms": 1e3, "second": 1e6, "s": 1e6}.get(units[ix[key]], 1.0)
+            elif sc is None:   # to GB
+                v *= {"byte": 1e-9, "Kbyte": 1e-6, "KB": 1e-6, "Mbyte": 1e-3, "MB": 1e-3, "Gbyte": 1.0, "GB": 1.0, "Tbyte": 1e3}.get(units[ix[key]], 1e-9)
             else:
                 v *= sc
             vals.append(f"{v:.3g}")
