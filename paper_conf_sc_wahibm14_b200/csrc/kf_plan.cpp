@@ -533,7 +533,7 @@ double model_time(const Program& p, const GroupLowering& L, const kf_target& t, 
     for (auto& st : p.kernels[k].stmts) ops += int(st.rpn.size()) + 1;
     work += (R / T) * (17.0 + 1.5 * ops);
   }
-  const int old_ctas = std::max(1, std::min(2048 / std::max(32, L.threads), 233472 / std::max(1, L.smem + 1024)));
+  const int old_ctas = std::max(1, std::min(2048 / std::max(32, L.threads), (t.smem_per_block + 1024) / std::max(1, L.smem + 1024)));
   const double old_eff = std::min(1.0, std::min(64.0, double(old_ctas) * (L.threads / 32)) / 32.0);
   const double t_comp = double(p.npts) * work / (2.5e13 * old_eff);
   const CanvasPlan cv = plan_canvas(p, L);
@@ -541,7 +541,10 @@ double model_time(const Program& p, const GroupLowering& L, const kf_target& t, 
   const double t_smem = double(p.npts) / T * per_plane / (128.0 * t.n_sm * 1.9e9);
   // resident warps
   const int need = int(32 * L.zunroll + 0.6 * (p.es / 4) * L.pts * (L.thrld + L.depth));
-  int ctas = std::max(1, std::min({233472 / std::max(1, L.smem + 1024), 2048 / std::max(32, L.threads), 32}));
+  // shared memory per SM = the per-CTA limit + the 1 KB reserve (B200: 232448 + 1024); scales with a
+  // hypothetical smem_per_block (the SMEM-capacity what-if of P:485)
+  const int smem_sm = t.smem_per_block + 1024;
+  int ctas = std::max(1, std::min({smem_sm / std::max(1, L.smem + 1024), 2048 / std::max(32, L.threads), 32}));
   while (ctas > 1 && regs_cap(L.threads, ctas) < need) ctas--;
   const bool pair = cv.ok && cv.pair;
   const double warps = double(ctas) * ((L.threads + 31) / 32) * (pair ? 2.0 : 1.0);
