@@ -433,7 +433,9 @@ AUTOTUNE_CANDIDATES = [  # (tile, stages, zunroll, ringunroll, minblocks, canvas
     ((32, 16, 43), 2, 1, 0, -1, 1, 2, 1), ((32, 16, 43), 2, 1, 0, -1, 1, 2, 0), ((64, 8, 43), 2, 1, 0, -1, 1, 2, 1),
     # three TMA stages for pairs: ncu showed 12 % of the flux group's warp samples waiting on the
     # mbarrier of the current plane (one plane of prefetch is not enough latency cover)
-    ((32, 8, 43), 3, 1, 0, -1, 1, 2, 1), ((32, 8, 43), 3, 1, 0, -1, 1, 2, 0), ((32, 8, 64), 3, 1, 0, -1, 1, 2, 1)]
+    ((32, 8, 43), 3, 1, 0, -1, 1, 2, 1), ((32, 8, 43), 3, 1, 0, -1, 1, 2, 0), ((32, 8, 64), 3, 1, 0, -1, 1, 2, 1),
+    # shorter / taller pair tiles: smaller planes make room for a third stage (4 rows), or less halo (12)
+    ((32, 4, 43), 3, 1, 0, -1, 1, 2, 1), ((32, 4, 43), 2, 1, 0, -1, 1, 2, 1), ((32, 12, 43), 2, 1, 0, -1, 1, 2, 1)]
 
 
 def cand_kw(base_kw, c):
