@@ -176,6 +176,7 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
     else
       o << "#ifndef KF_CAP\n#define KF_BOUNDS " << primary << "\n#else\n#define KF_BOUNDS __maxnreg__(KF_CAP)\n#endif\n";
   }
+  o << "/*@@KF_GCOPY@@*/";
   o << "extern \"C\" __global__ void KF_BOUNDS " << cg.name << "(const __grid_constant__ KfArgs a) {\n";
   // pointer arithmetic from the __shared__ array keeps the shared state space (LDS/STS, 32-bit
   // addressing); the pad realigns the dynamic window to 128 bytes (TMA destinations).
@@ -919,8 +920,65 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
   for (const Ring& R : L.rings) rot_slots += R.slots > 1 ? R.slots : 0;
   const bool rotate = rot_slots <= 32 && !getenv("KF_SLOT_COUNTERS");   // A/B switch: per-ring counters + kf_slot
   if (getenv("KF_DEBUG")) fprintf(stderr, "codegen %s: %d rotated ring slots%s\n", cg.name.c_str(), rot_slots, rotate ? "" : " (counters)");
+  // Periodic ghost copies written by the producer (ghostwrite; no ghost-fill launches): at the start
+  // of iteration t an edge tile copies, for every live-out, the points it stored in the previous
+  // iteration (plane tt - D_k + uu of its producer k) within the ghost width of a periodic x / y
+  // boundary to the opposite ghost layer (corners too).  The values are re-read from global memory
+  // (written by this CTA before the end-of-iteration barrier, still in L2), off the compute path and
+  // outside its registers.  x images are whole 32-byte sectors when the row origin and NX allow it
+  // (a ghost span widened into the padding: no partial-sector stores, which cost the L2 an ECC
+  // read-modify-write -- ncu, round 2).
+  const bool ghost_copy_on = L.ghost_write && !L.live_out.empty();
+  const int ESEC = 32 / es;
+  const bool xsector = lay.xoff >= ESEC && p.ghost[0] <= ESEC && NX % ESEC == 0 && (lay.xoff * es) % 32 == 0 &&
+                       (lay.pitch * es) % 32 == 0;
+  auto emit_ghost_copy_body = [&](std::ostream& o, const std::string& tt, const std::string& ind) {
+    const bool px_ = p.bc[0] == KF_BC_PERIODIC, py_ = p.bc[1] == KF_BC_PERIODIC;
+    const std::string EX = xsector ? std::to_string(ESEC) : "GX";
+    o << ind << "{ const int tw = min(TX, NX - x0), th = min(TY, NY - y0);\n";
+    o << ind << "  const int xa0 = x0, xa1 = " << (px_ ? "min(" + EX + ", x0 + tw)" : "x0") << ";\n";
+    o << ind << "  const int xb0 = " << (px_ ? "max(NX - " + EX + ", x0 + max(xa1 - x0, 0))" : "x0 + tw") << ", xb1 = x0 + tw;\n";
+    o << ind << "  const int ya0 = y0, ya1 = " << (py_ ? "min(GY, y0 + th)" : "y0") << ";\n";
+    o << ind << "  const int yb0 = " << (py_ ? "max(NY - GY, y0 + max(ya1 - y0, 0))" : "y0 + th") << ", yb1 = y0 + th;\n";
+    o << ind << "  const int na = max(xa1 - xa0, 0), nb = max(xb1 - xb0, 0), ncx = na + nb;\n";
+    o << ind << "  const int nya = max(ya1 - ya0, 0), ncy = nya + max(yb1 - yb0, 0);\n";
+    o << ind << "  const int per = ncx * th + (tw - ncx) * ncy;   // x strips (all rows), then y strips (other columns)\n";
+    o << ind << "  #pragma unroll 1\n";
+    o << ind << "  for (int i = tid; i < per * " << U << "; i += NT) {\n";
+    o << ind << "    const int uu = i / per, r = i - uu * per;\n";
+    o << ind << "    int gx, gy;\n";
+    o << ind << "    if (r < ncx * th) { const int c = r / th; gy = y0 + (r - c * th); gx = c < na ? xa0 + c : xb0 + (c - na); }\n";
+    o << ind << "    else { const int q = r - ncx * th, w = tw - ncx, c = q / w;   // columns [x0 + na, x0 + tw - nb)\n";
+    o << ind << "           gy = c < nya ? ya0 + c : yb0 + (c - nya); gx = x0 + na + (q - c * w); }\n";
+    o << ind << "    const bool wx = " << (px_ ? "(gx < " + EX + " || gx >= NX - " + EX + ")" : "false") << ", wy = "
+      << (py_ ? "(gy < GY || gy >= NY - GY)" : "false") << ";\n";
+    o << ind << "    const int gx2 = gx < " << EX << " ? gx + NX : gx - NX, gy2 = gy < GY ? gy + NY : gy - NY;\n";
+    for (size_t oi = 0; oi < L.live_out.size(); oi++) {
+      const Ver v = L.live_out[oi];
+      const int k = p.writer_of(v.x, v.v);
+      o << ind << "    { const int pz = " << tt << " - " << L.delay.at(k) << " + uu;\n";
+      o << ind << "      if (pz >= z0 && pz < z1) {\n";
+      o << ind << "        const long long pb = (long long)pz * PLANE;\n";
+      o << ind << "        const real v = a.out[" << oi << "][pb + (long long)gy * PITCH + gx];\n";
+      o << ind << "        if (wx) a.out[" << oi << "][pb + (long long)gy * PITCH + gx2] = v;\n";
+      o << ind << "        if (wy) a.out[" << oi << "][pb + (long long)gy2 * PITCH + gx] = v;\n";
+      o << ind << "        if (wx && wy) a.out[" << oi << "][pb + (long long)gy2 * PITCH + gx2] = v;\n";
+      o << ind << "      }\n    }\n";
+    }
+    o << ind << "  }\n" << ind << "}\n";
+  };
+  // the copy is a __noinline__ function (emitted before the kernel): inlined into the stream loop it
+  // raised a flux group from 127 to 204 registers
+  auto emit_ghost_copy = [&](const std::string& tt, const std::string& ind) {
+    o << ind << "kf_gcopy(a, " << tt << ", x0, y0, z0, z1);\n";
+  };
   auto emit_body = [&](int j) {
   o << "    if (tid == 0 && t + " << U << " * (NSTAGE - 1) < t1) issue(t + " << U << " * (NSTAGE - 1));\n";
+  if (ghost_copy_on) {
+    o << "    if (edge_tile && t > t0) {\n";
+    emit_ghost_copy("(t - " + std::to_string(U) + ")", "      ");
+    o << "    }\n";
+  }
   o << "    kf_mbar_wait(&mbar[((t - t0) / " << U << ") % NSTAGE], (((t - t0) / " << U << ") / NSTAGE) & 1);\n";
 
   auto mid_index = [&](int ring) {
@@ -1340,6 +1398,7 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
   }
   if (use_canvas) o << "    }\n";
   o << "    __syncthreads();\n";
+  if (ghost_copy_on) o << "    t_prev = t;\n";
   if (NU != 0)
     for (auto& [ring, om] : undefs) o << "#undef P" << ring << "_" << om << "\n";
   };   // emit_body
@@ -1362,6 +1421,7 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
       for (auto& [key, src] : carry) o << "  real " << key_name("cq", key, "_r" + std::to_string(r)) << " = 0;\n";
   }
   o << canvas_bounds;
+  if (ghost_copy_on) o << "  int t_prev = t0 - 1;   // the last stream iteration run (ghost copies of its planes follow the loop)\n";
   if (NU == 0 && rotate) {
     // slot byte offsets of every ring, rotated by U slots per iteration: slot (c + om) mod n of a
     // per-ring counter c costs ~5 uniform instructions per pointer and iteration (ncu: ~35 % of all
@@ -1399,42 +1459,26 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
     }
     o << "  }\n";
   }
-  // Periodic ghost copies of the live-outs (ghostwrite): after its whole z range, an edge tile copies
-  // the points it stored within the ghost width of a periodic x/y boundary to the opposite ghost
-  // layer (corners too), so the step needs no ghost-fill launches.  A separate epilogue keeps these
-  // scattered stores out of the compute loop's register budget; the values are re-read from global
-  // memory, written by this CTA before the barrier.
-  if (L.ghost_write && !L.live_out.empty()) {
-    const bool px_ = p.bc[0] == KF_BC_PERIODIC, py_ = p.bc[1] == KF_BC_PERIODIC;
-    o << "  if (edge_tile) {\n";
-    o << "    __syncthreads();\n";
-    o << "    const int tw = min(TX, NX - x0), th = min(TY, NY - y0), tzn = z1 - z0;\n";
-    // column strips (x) and row strips (y) of the tile inside the ghost width of a periodic boundary
-    o << "    const int xa0 = x0, xa1 = " << (px_ ? "min(GX, x0 + tw)" : "x0") << ";\n";
-    o << "    const int xb0 = " << (px_ ? "max(NX - GX, x0 + (xa1 > x0 ? xa1 - x0 : 0))" : "x0 + tw") << ", xb1 = x0 + tw;\n";
-    o << "    const int ya0 = y0, ya1 = " << (py_ ? "min(GY, y0 + th)" : "y0") << ";\n";
-    o << "    const int yb0 = " << (py_ ? "max(NY - GY, y0 + (ya1 > y0 ? ya1 - y0 : 0))" : "y0 + th") << ", yb1 = y0 + th;\n";
-    o << "    const int ncx = max(xa1 - xa0, 0) + max(xb1 - xb0, 0), ncy = max(ya1 - ya0, 0) + max(yb1 - yb0, 0);\n";
-    o << "    const int per = ncx * th + tw * ncy;\n";
-    o << "    for (int i = tid; i < per * tzn; i += NT) {\n";
-    o << "      const int zz = i / per, r = i - zz * per;\n";
-    o << "      int gx, gy;\n";
-    o << "      if (r < ncx * th) { const int c = r / th; gy = y0 + (r - c * th); gx = c < max(xa1 - xa0, 0) ? xa0 + c : xb0 + c - max(xa1 - xa0, 0); }\n";
-    o << "      else { const int q = r - ncx * th, c = q / tw; gx = x0 + (q - c * tw); gy = c < max(ya1 - ya0, 0) ? ya0 + c : yb0 + c - max(ya1 - ya0, 0); }\n";
-    o << "      const bool wx = " << (px_ ? "(gx < GX || gx >= NX - GX)" : "false") << ", wy = "
-      << (py_ ? "(gy < GY || gy >= NY - GY)" : "false") << ";\n";
-    o << "      const int gx2 = gx < GX ? gx + NX : gx - NX, gy2 = gy < GY ? gy + NY : gy - NY;\n";
-    o << "      const long long pb = (long long)(z0 + zz) * PLANE;\n";
-    for (size_t oi = 0; oi < L.live_out.size(); oi++) {
-      o << "      { const real v = a.out[" << oi << "][pb + (long long)gy * PITCH + gx];\n";
-      o << "        if (wx) a.out[" << oi << "][pb + (long long)gy * PITCH + gx2] = v;\n";
-      o << "        if (wy) a.out[" << oi << "][pb + (long long)gy2 * PITCH + gx] = v;\n";
-      o << "        if (wx && wy) a.out[" << oi << "][pb + (long long)gy2 * PITCH + gx2] = v; }\n";
-    }
-    o << "    }\n  }\n";
+  if (ghost_copy_on) {
+    o << "  __syncthreads();\n";
+    o << "  if (edge_tile && t_prev >= t0) {\n";
+    emit_ghost_copy("t_prev", "    ");
+    o << "  }\n";
   }
   o << "}\n";
   cg.source = o.str();
+  {
+    std::ostringstream fo;
+    if (ghost_copy_on) {
+      fo << "static __device__ __noinline__ void kf_gcopy(const KfArgs& a, const int tt, const int x0, const int y0,"
+            " const int z0, const int z1) {\n  const int tid = threadIdx.x;\n";
+      emit_ghost_copy_body(fo, "tt", "  ");
+      fo << "}\n";
+    }
+    const std::string mark = "/*@@KF_GCOPY@@*/";
+    const size_t at = cg.source.find(mark);
+    if (at != std::string::npos) cg.source.replace(at, mark.size(), fo.str());
+  }
   {
     const std::string mark = "/*@@KF_CLAMP_BASES@@*/";
     for (size_t at = cg.source.find(mark); at != std::string::npos; at = cg.source.find(mark, at))

@@ -106,7 +106,18 @@ static Compiled nvrtc_compile(const std::string& src, const std::string& name) {
   if (ls) nvrtcGetProgramLog(prog, &c.log[0]);
   if (r != NVRTC_SUCCESS) {
     nvrtcDestroyProgram(&prog);
-    fail(KF_E_NVRTC, "NVRTC failed for " + name + ": " + c.log.substr(0, 4000));
+    // the errors, not the warnings, first
+    std::string errs;
+    for (size_t a = 0, b; a < c.log.size(); a = b + 1) {
+      b = c.log.find('\n', a);
+      if (b == std::string::npos) b = c.log.size();
+      const std::string line = c.log.substr(a, b - a);
+      if (line.find("error") != std::string::npos) errs += line + "\n";
+    }
+    if (const char* dir = getenv("KF_DUMP_DIR")) {
+      if (FILE* f = fopen((std::string(dir) + "/" + name + "_failed.cu").c_str(), "w")) { fwrite(src.data(), 1, src.size(), f); fclose(f); }
+    }
+    fail(KF_E_NVRTC, "NVRTC failed for " + name + ": " + errs.substr(0, 3000) + c.log.substr(0, 1000));
   }
   size_t cs = 0;
   nvrtcGetCUBINSize(prog, &cs);
