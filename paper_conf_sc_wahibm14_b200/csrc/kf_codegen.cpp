@@ -920,19 +920,17 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
   for (const Ring& R : L.rings) rot_slots += R.slots > 1 ? R.slots : 0;
   const bool rotate = rot_slots <= 32 && !getenv("KF_SLOT_COUNTERS");   // A/B switch: per-ring counters + kf_slot
   if (getenv("KF_DEBUG")) fprintf(stderr, "codegen %s: %d rotated ring slots%s\n", cg.name.c_str(), rot_slots, rotate ? "" : " (counters)");
-  // Periodic ghost copies written by the producer (ghostwrite; no ghost-fill launches): at the start
-  // of iteration t an edge tile copies, for every live-out, the points it stored in the previous
-  // iteration (plane tt - D_k + uu of its producer k) within the ghost width of a periodic x / y
-  // boundary to the opposite ghost layer (corners too).  The values are re-read from global memory
-  // (written by this CTA before the end-of-iteration barrier, still in L2), off the compute path and
-  // outside its registers.  x images are whole 32-byte sectors when the row origin and NX allow it
-  // (a ghost span widened into the padding: no partial-sector stores, which cost the L2 an ECC
-  // read-modify-write -- ncu, round 2).
+  // Periodic ghost copies written by the producer (ghostwrite; no ghost-fill launches): after its z
+  // loop an edge tile copies, for every live-out and plane it stored, the points within the ghost
+  // width of a periodic x / y boundary to the opposite ghost layer (corners too), re-reading them
+  // from global memory (written by this CTA before the barrier).  x images are whole 32-byte
+  // sectors when the row origin and NX allow it (a ghost span widened into the padding: no
+  // partial-sector stores, which cost the L2 an ECC read-modify-write -- ncu, round 2).
   const bool ghost_copy_on = L.ghost_write && !L.live_out.empty();
   const int ESEC = 32 / es;
   const bool xsector = lay.xoff >= ESEC && p.ghost[0] <= ESEC && NX % ESEC == 0 && (lay.xoff * es) % 32 == 0 &&
                        (lay.pitch * es) % 32 == 0;
-  auto emit_ghost_copy_body = [&](std::ostream& o, const std::string& tt, const std::string& ind) {
+  auto emit_ghost_copy_body = [&](std::ostream& o, const std::string& tt, const std::string& ind, bool delays) {
     const bool px_ = p.bc[0] == KF_BC_PERIODIC, py_ = p.bc[1] == KF_BC_PERIODIC;
     const std::string EX = xsector ? std::to_string(ESEC) : "GX";
     o << ind << "{ const int tw = min(TX, NX - x0), th = min(TY, NY - y0);\n";
@@ -956,7 +954,7 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
     for (size_t oi = 0; oi < L.live_out.size(); oi++) {
       const Ver v = L.live_out[oi];
       const int k = p.writer_of(v.x, v.v);
-      o << ind << "    { const int pz = " << tt << " - " << L.delay.at(k) << " + uu;\n";
+      o << ind << "    { const int pz = " << tt << " - " << (delays ? L.delay.at(k) : 0) << " + uu;\n";
       o << ind << "      if (pz >= z0 && pz < z1) {\n";
       o << ind << "        const long long pb = (long long)pz * PLANE;\n";
       o << ind << "        const real v = a.out[" << oi << "][pb + (long long)gy * PITCH + gx];\n";
@@ -967,18 +965,11 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
     }
     o << ind << "  }\n" << ind << "}\n";
   };
-  // the copy is a __noinline__ function (emitted before the kernel): inlined into the stream loop it
-  // raised a flux group from 127 to 204 registers
-  auto emit_ghost_copy = [&](const std::string& tt, const std::string& ind) {
-    o << ind << "kf_gcopy(a, " << tt << ", x0, y0, z0, z1);\n";
-  };
+  // the copy is a __noinline__ function (emitted before the kernel), called per plane by edge tiles
+  // after their z loop
   auto emit_body = [&](int j) {
   o << "    if (tid == 0 && t + " << U << " * (NSTAGE - 1) < t1) issue(t + " << U << " * (NSTAGE - 1));\n";
-  if (ghost_copy_on) {
-    o << "    if (edge_tile && t > t0) {\n";
-    emit_ghost_copy("(t - " + std::to_string(U) + ")", "      ");
-    o << "    }\n";
-  }
+
   o << "    kf_mbar_wait(&mbar[((t - t0) / " << U << ") % NSTAGE], (((t - t0) / " << U << ") / NSTAGE) & 1);\n";
 
   auto mid_index = [&](int ring) {
@@ -1398,7 +1389,6 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
   }
   if (use_canvas) o << "    }\n";
   o << "    __syncthreads();\n";
-  if (ghost_copy_on) o << "    t_prev = t;\n";
   if (NU != 0)
     for (auto& [ring, om] : undefs) o << "#undef P" << ring << "_" << om << "\n";
   };   // emit_body
@@ -1421,7 +1411,7 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
       for (auto& [key, src] : carry) o << "  real " << key_name("cq", key, "_r" + std::to_string(r)) << " = 0;\n";
   }
   o << canvas_bounds;
-  if (ghost_copy_on) o << "  int t_prev = t0 - 1;   // the last stream iteration run (ghost copies of its planes follow the loop)\n";
+
   if (NU == 0 && rotate) {
     // slot byte offsets of every ring, rotated by U slots per iteration: slot (c + om) mod n of a
     // per-ring counter c costs ~5 uniform instructions per pointer and iteration (ncu: ~35 % of all
@@ -1460,9 +1450,11 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
     o << "  }\n";
   }
   if (ghost_copy_on) {
+    // after the whole z range (round 2: per-iteration copies, even in a __noinline__ function, made
+    // every group 10-30 % slower; the epilogue 5-15 %; the fills are the default)
     o << "  __syncthreads();\n";
-    o << "  if (edge_tile && t_prev >= t0) {\n";
-    emit_ghost_copy("t_prev", "    ");
+    o << "  if (edge_tile) {\n";
+    o << "    for (int tz = z0; tz < z1; tz += " << U << ") kf_gcopy(a, tz, x0, y0, z0, z1);\n";
     o << "  }\n";
   }
   o << "}\n";
@@ -1472,7 +1464,7 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
     if (ghost_copy_on) {
       fo << "static __device__ __noinline__ void kf_gcopy(const KfArgs& a, const int tt, const int x0, const int y0,"
             " const int z0, const int z1) {\n  const int tid = threadIdx.x;\n";
-      emit_ghost_copy_body(fo, "tt", "  ");
+      emit_ghost_copy_body(fo, "tt", "  ", false);
       fo << "}\n";
     }
     const std::string mark = "/*@@KF_GCOPY@@*/";
