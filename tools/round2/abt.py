@@ -5,7 +5,8 @@ the step time and of every group's time.
   python tools/round2/abt.py '<json spec>'
   spec = {"workload": "weather", "plan": [...labels], "tuned": [[tile, stages, zunroll, ringunroll,
           minblocks, canvas_ld, pblock_x, pair_zq], ...], "variants": [{"name": .., "ghostwrite": 0|1,
-          "override": {group: [...config]}, "env": {..}}], "rounds": 5, "steps": 10}
+          "override": {group: [...config]}, "env": {..},
+          "target": {kf_target field: value}}], "rounds": 5, "steps": 10}
 """
 import json
 import os
@@ -40,6 +41,7 @@ def main():
             old[k] = os.environ.get(k)
             os.environ[k] = str(val)
         base = dict(wl.tkw, ghostwrite=v.get("ghostwrite", 1))
+        base.update(v.get("target", {}))   # e.g. {"wrapload": 1}
         gt = [kf.Target(**bench.cand_kw(base, c)) for c in tuned]
         ex = kf.Exec(prog, plan, gt[0], group_targets=gt)
         for k, o in old.items():
