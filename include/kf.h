@@ -187,15 +187,8 @@ typedef struct {
   int32_t pair_zq;               /* pair canvas (pblock 2x1): 1 = z-column values carried in
                                     registers across stream iterations instead of re-read
                                     from shared memory (more registers), 0 = off             */
-  int32_t wrapload;              /* 1: on a single domain with periodic x and y (R9, P:82 padding),
-                                    tiles whose staged boxes cross the domain edge load the
-                                    wrapped parts from the opposite side themselves (one bulk
-                                    copy per box row segment instead of the tiled TMA box), so
-                                    a step launches no periodic ghost fills; 0 = ghost fills.
-                                    Ignored (fills) with ghostwrite, internal axes, or a
-                                    periodic x whose row NX*es is not a multiple of 16 bytes */
 } kf_target;
-/* Fills the B200 defaults: 8.0e12, 232448, 255, 148, {64,4,0}, 2, 256, 16, 0, 1, {1,1}, 0, 0, 0, 0, 1, 1, 0. */
+/* Fills the B200 defaults: 8.0e12, 232448, 255, 148, {64,4,0}, 2, 256, 16, 0, 1, {1,1}, 0, 0, 0, 0, 1, 1. */
 kf_status kf_target_b200(kf_target* out);
 
 /* ------------------------------------------------------------------ legality (Eq. 1.1-1.7) */

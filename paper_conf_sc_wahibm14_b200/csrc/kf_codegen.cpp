@@ -94,10 +94,6 @@ static __device__ __forceinline__ void kf_tma_load3(void* dst, const KfTmap* map
   asm volatile("cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], [%5];"
                :: "r"(kf_smem_u32(dst)), "l"((u64)map), "r"(c0), "r"(c1), "r"(c2), "r"(kf_smem_u32(m)) : "memory");
 }
-static __device__ __forceinline__ void kf_bulk_load(void* dst, const void* src, u32 bytes, u64* m) {
-  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
-               :: "r"(kf_smem_u32(dst)), "l"(src), "r"(bytes), "r"(kf_smem_u32(m)) : "memory");
-}
 static __device__ __forceinline__ int kf_mod(int a, int m) { int r = a % m; return r < 0 ? r + m : r; }
 static __device__ __forceinline__ int kf_slot(int c, int om, int n) { int s = c + om; return s >= n ? s - n : s; }
 )KF";
@@ -144,47 +140,7 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
   o << "  const real* gsrc[" << std::max<size_t>(1, mid_rings.size()) << "];\n";
   o << "  double prm[" << std::max(1, p.n_params) << "];\n";
   o << "  int mode, pad_;   // units: 0 all, 1 interior tiles only, 2 the others (kf_split_units)\n";
-  o << "  const real* gin[" << std::max<size_t>(1, in_rings.size()) << "];   // live-in buffers (wrapped row loads)\n";
   o << "};\n";
-  // Wrapped loads (kf_target.wrapload, R9 periodic axes): a box that crosses the domain edge on a
-  // periodic axis is loaded row by row with 1D bulk copies (cp.async.bulk, same mbarrier and byte
-  // count as the TMA box), each row split where it crosses x = 0 or NX and its source wrapped to the
-  // opposite side; rows wrap in y, the plane in z (periodic z).  Every segment starts and ends on a
-  // 16-byte boundary: box starts are 16-byte aligned (ax_lo), NX*es is a multiple of 16 (lowering).
-  if (L.wrap_axes) {
-    o << "static __device__ __forceinline__ void kf_rows(unsigned char* dst, const real* g, int xs, int ys, int P, int W, int H,\n"
-      << "                                               bool wx, bool wy, int lane, int nl, u64* mb) {\n"
-      << "  for (int r = lane; r < H; r += nl) {\n"
-      << "    const int gy = wy ? kf_mod(ys + r, NY) : ys + r;\n"
-      << "    const real* row = g + (long long)(GZ + P) * PLANE + (long long)(GY + gy) * PITCH + XOFF;\n"
-      << "    unsigned char* d = dst + r * W * (int)sizeof(real);\n"
-      << "    int x = xs, rem = W;\n"
-      << "    while (rem > 0) {\n"
-      << "      const int sx = wx ? kf_mod(x, NX) : x;\n"
-      << "      const int n = wx ? min(rem, NX - sx) : rem;\n"
-      << "      kf_bulk_load(d, row + sx, (u32)(n * (int)sizeof(real)), mb);\n"
-      << "      d += n * (int)sizeof(real); x += n; rem -= n;\n"
-      << "    }\n  }\n}\n";
-    // every wrapped box of one stream iteration from ONE call site (a __noinline__ function: the
-    // stream loop keeps its registers; bit ti*U+uu = ring ti, plane t+uu+A)
-    const int U = L.zunroll;
-    o << "static __device__ __noinline__ void kf_wrap_rows(const KfArgs* a, unsigned char* sm, u32 rowm, int t, int t0, int x0,\n"
-      << "                                                 int y0, int lane, u64* mb) {\n";
-    int ti = 0;
-    for (int ri : in_rings) {
-      const Ring& r = L.rings[ri];
-      for (int uu = 0; uu < U; uu++) {
-        const std::string P = "(t + " + std::to_string(uu + r.A) + ")";
-        const std::string pz = (L.wrap_axes & 4) ? "kf_mod(" + P + ", NZ)" : P;
-        o << "  if (rowm & " << (1u << (ti * U + uu)) << "u) kf_rows(sm + " << r.smem_off << " + kf_mod(" << P << " - t0, "
-          << r.slots << ") * " << r.plane_bytes << ", a->gin[" << ti << "], x0 - " << r.ax_lo << ", y0 - " << r.blo[1] << ", "
-          << pz << ", " << r.px << ", " << r.hy << ", x0 - " << r.ax_lo << " < 0 || x0 - " << r.ax_lo << " + " << r.px
-          << " > NX, y0 - " << r.blo[1] << " < 0 || y0 - " << r.blo[1] << " + " << r.hy << " > NY, lane, 32, mb);\n";
-      }
-      ti++;
-    }
-    o << "}\n";
-  }
   // Registers.  minblocks -1: __launch_bounds__(NT), ptxas' own choice (measured: explicit budgets
   // make ptxas use up to the budget, e.g. 124 or 162 instead of 88 or 72 registers on the flux
   // groups, one CTA per SM less).  minblocks >= 0: __maxnreg__ at what keeps m CTAs per SM resident
@@ -256,20 +212,6 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
   o << "  const int z1 = min(z0 + TZ, NZ);\n";
   o << "  const bool edge_tile = x0 < GX || x0 + TX > NX - GX || y0 < GY || y0 + TY > NY - GY;\n";
   o << "  if (tid == 0) {\n    for (int s = 0; s < NSTAGE; ++s) kf_mbar_init(&mbar[s], 1);\n    kf_fence_init();\n  }\n";
-  // wrapped loads: which live-in boxes of this tile cross the domain edge (then warp 0 issues the
-  // row copies of the tile; other tiles keep one TMA box per ring, issued by thread 0)
-  if (L.wrap_axes) {
-    // bit 2r: ring r's box crosses x = 0 or NX; bit 2r+1: y = 0 or NY (one register for the tile)
-    o << "  u32 wrap_mask = 0u;\n";
-    for (size_t i = 0; i < in_rings.size(); i++) {
-      const Ring& r = L.rings[in_rings[i]];
-      o << "  if (x0 - " << r.ax_lo << " < 0 || x0 - " << r.ax_lo << " + " << r.px << " > NX) wrap_mask |= " << (1u << (2 * i)) << "u;\n";
-      o << "  if (y0 - " << r.blo[1] << " < 0 || y0 - " << r.blo[1] << " + " << r.hy << " > NY) wrap_mask |= " << (2u << (2 * i)) << "u;\n";
-    }
-    o << "  const bool wrap_cta = wrap_mask != 0u;\n";
-  } else {
-    o << "  const bool wrap_cta = false;\n";
-  }
   // per-kernel starting point of the thread in its region (row-major, x fastest)
   for (int k : alive) {
     const Ext& e = L.ext.at(k);
@@ -440,39 +382,18 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
       o << "    if (ok" << ri << "_" << uu << ") bytes += " << (r.px * r.hy * es) << "u;\n";
     }
   }
-  // called by thread 0, or by warp 0 on tiles with wrapped boxes: lane 0 arms the barrier and
-  // issues the TMA boxes, every lane a share of the row copies.  No __syncwarp: a copy that
-  // completes before lane 0's arrive.expect_tx leaves the tx-count negative, and the phase cannot
-  // complete before that arrive (the barrier counts one arrival).  The mask is re-read through an
-  // opaque move so the per-ring tests are not hoisted into loop-carried registers.
-  o << "    if (tid == 0) kf_mbar_expect(mb, bytes);\n";
-  if (L.wrap_axes) o << "    u32 wm, rowm = 0u;\n    asm volatile(\"mov.b32 %0, %1;\" : \"=r\"(wm) : \"r\"(wrap_mask));\n";
+  o << "    kf_mbar_expect(mb, bytes);\n";
   int ti = 0;
-  const std::string zw = (L.wrap_axes & 4) ? "kf_mod(P%, NZ)" : "P%";
   for (int ri : in_rings) {
     const Ring& r = L.rings[ri];
-    for (int uu = 0; uu < U; uu++) {
-      const std::string pv = std::to_string(ri) + "_" + std::to_string(uu);
-      std::string pz = zw;
-      pz.replace(pz.find('%'), 1, pv);
-      const std::string dst = "sm + " + std::to_string(r.smem_off) + " + kf_mod(P" + pv + " - t0, " + std::to_string(r.slots) +
-                              ") * " + std::to_string(r.plane_bytes);
-      if (L.wrap_axes) {
-        o << "    if (ok" << pv << ") {\n";
-        o << "      if ((wm >> " << 2 * ti << ") & 3u) rowm |= " << (1u << (ti * U + uu)) << "u;\n";
-        o << "      else if (tid == 0) kf_tma_load3(" << dst << ", &a.tm[" << ti << "], XOFF + x0 - (" << r.ax_lo
-          << "), GY + y0 - (" << r.blo[1] << "), GZ + " << pz << ", mb);\n";
-        o << "    }\n";
-      } else {
-        o << "    if (ok" << pv << ") kf_tma_load3(" << dst << ", &a.tm[" << ti << "], XOFF + x0 - (" << r.ax_lo
-          << "), GY + y0 - (" << r.blo[1] << "), GZ + " << pz << ", mb);\n";
-      }
-    }
+    for (int uu = 0; uu < U; uu++)
+      o << "    if (ok" << ri << "_" << uu << ") kf_tma_load3(sm + " << r.smem_off << " + kf_mod(P" << ri << "_" << uu << " - t0, "
+        << r.slots << ") * " << r.plane_bytes << ", &a.tm[" << ti << "], XOFF + x0 - (" << r.ax_lo << "), GY + y0 - ("
+        << r.blo[1] << "), GZ + P" << ri << "_" << uu << ", mb);\n";
     ti++;
   }
-  if (L.wrap_axes) o << "    if (rowm) kf_wrap_rows(&a, sm, rowm, t, t0, x0, y0, tid, mb);\n";
   o << "  };\n";
-  o << "  if (tid == 0 || (wrap_cta && tid < 32))\n    for (int t = t0; t < t1 && t < t0 + " << U << " * (NSTAGE - 1); t += " << U << ") issue(t);\n";
+  o << "  if (tid == 0)\n    for (int t = t0; t < t1 && t < t0 + " << U << " * (NSTAGE - 1); t += " << U << ") issue(t);\n";
   // Ring slots are relative to the CTA's first iteration: plane P lives in slot (P - t0) mod n.
   // With ring unrolling (every ring size a power of two dividing N) the loop body is emitted N
   // times and every slot is a compile-time constant: no per-iteration pointer arithmetic.
@@ -1047,7 +968,7 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
   // the copy is a __noinline__ function (emitted before the kernel), called per plane by edge tiles
   // after their z loop
   auto emit_body = [&](int j) {
-  o << "    if ((tid == 0 || (wrap_cta && tid < 32)) && t + " << U << " * (NSTAGE - 1) < t1) issue(t + " << U << " * (NSTAGE - 1));\n";
+  o << "    if (tid == 0 && t + " << U << " * (NSTAGE - 1) < t1) issue(t + " << U << " * (NSTAGE - 1));\n";
 
   o << "    kf_mbar_wait(&mbar[((t - t0) / " << U << ") % NSTAGE], (((t - t0) / " << U << ") / NSTAGE) & 1);\n";
 

@@ -135,7 +135,6 @@ struct GroupLowering {
   int ring_unroll = 0;      // 0, or N: every ring size a power of two dividing N, loop unrolled N times
   bool ghost_write = false; // live-out stores also write the periodic x/y ghost copies (no fills)
   int pair_zq = 1;          // pair canvas: z-column register queues (kf_target.pair_zq)
-  int wrap_axes = 0;        // axes whose live-in boxes the kernel loads wrapped (kf_target.wrapload)
   int canvas_ld = 1;        // fast-iteration shared loads unpredicated where in bounds (kf_target.canvas_ld)
   int minblocks = 0;        // __launch_bounds__ min CTAs/SM: 0 auto (SMEM-limited), -1 none, n
   int ring_of(const Ver& v) const;        // index in rings or -1

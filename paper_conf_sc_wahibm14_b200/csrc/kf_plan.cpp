@@ -84,10 +84,6 @@ GroupLowering lower_group(const Program& p, const std::vector<int>& g, const kf_
   L.minblocks = t.minblocks;
   L.canvas_ld = t.canvas_ld;
   L.pair_zq = t.pair_zq;
-  // wrapped loads (kf_target.wrapload): a single domain, periodic x and y, 16-byte row segments
-  if (t.wrapload && !L.ghost_write && !(t.internal_axes & 3) && p.bc[0] == KF_BC_PERIODIC &&
-      p.bc[1] == KF_BC_PERIODIC && (p.n[0] * p.es) % 16 == 0)
-    L.wrap_axes = 3 | (p.bc[2] == KF_BC_PERIODIC && !(t.internal_axes & 4) ? 4 : 0);
   L.pblock[0] = t.pblock[0];
   L.pblock[1] = t.pblock[1];
   L.live_in = group_live_in(p, g);
@@ -310,12 +306,6 @@ GroupLowering lower_group(const Program& p, const std::vector<int>& g, const kf_
     L.regs = 32 * U + (es / 4) * P * (thrld + depth);
     L.thrld = thrld;
     L.pts = P;
-  }
-  // wrapped loads: one bit per (live-in ring, plane of the stream iteration) in a u32 mask
-  if (L.wrap_axes) {
-    int nin = 0;
-    for (const Ring& r : L.rings) nin += r.live_in ? 1 : 0;
-    if (nin * L.zunroll > 32) L.wrap_axes = 0;
   }
   return L;
 }
@@ -580,7 +570,6 @@ void check_target(const kf_target* t) {
   if (t->skew < 0 || t->skew > 1) fail(KF_E_ARG, "skew must be 0 or 1");
   if (t->canvas_ld < 0 || t->canvas_ld > 1) fail(KF_E_ARG, "canvas_ld must be 0 or 1");
   if (t->pair_zq < 0 || t->pair_zq > 1) fail(KF_E_ARG, "pair_zq must be 0 or 1");
-  if (t->wrapload < 0 || t->wrapload > 1) fail(KF_E_ARG, "wrapload must be 0 or 1");
   if (t->pblock[0] < 1 || t->pblock[0] > 4 || t->pblock[1] < 1 || t->pblock[1] > 4)
     fail(KF_E_ARG, "pblock must be in [1, 4] x [1, 4]");
   if (t->threads < 32 || t->threads > 1024 || t->threads % 32) fail(KF_E_ARG, "threads must be a multiple of 32 in [32,1024]");

@@ -358,8 +358,6 @@ kf_status kf_target_b200(kf_target* out) {
     t.skew = 0;
     t.canvas_ld = 1;
     t.pair_zq = 1;
-    t.wrapload = 0;
-    if (const char* w = getenv("KF_WRAPLOAD")) t.wrapload = atoi(w) ? 1 : 0;   // A/B switch for test sweeps
     *out = t;
   });
 }

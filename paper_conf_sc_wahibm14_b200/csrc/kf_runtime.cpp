@@ -338,7 +338,7 @@ static void build_blobs(kf_exec* E) {
     for (auto& g : E->G) {
       size_t ni = std::max<size_t>(1, g.ins.size()), no = std::max<size_t>(1, g.outs.size()),
              nm = std::max<size_t>(1, g.mids.size()), np = std::max(1, p.n_params);
-      size_t sz = 128 * ni + 8 * (no + nm + np) + 8 + 8 * ni;   // + int mode, pad (zero: every unit), gin[]
+      size_t sz = 128 * ni + 8 * (no + nm + np) + 8;   // + int mode, pad (zero: every unit)
       sz = (sz + 63) / 64 * 64;
       g.blob_size = sz;
       std::vector<unsigned char> b(sz + 64, 0);
@@ -374,11 +374,6 @@ static void build_blobs(kf_exec* E) {
       }
       q += 8 * nm;
       for (int j = 0; j < p.n_params; j++) std::memcpy(q + 8 * j, &E->cur_params[j], 8);
-      q += 8 * np + 8;   // int mode, pad_
-      for (size_t i = 0; i < g.ins.size(); i++) {   // gin[]: the live-in buffers (wrapped row loads)
-        void* ptr = buf_ptr(E, buffer_id(E, g.ins[i], par));
-        std::memcpy(q + 8 * i, &ptr, 8);
-      }
       std::vector<unsigned char> out(base, base + sz);
       E->blobs[par][&g - &E->G[0]] = std::move(out);
     }
@@ -509,8 +504,8 @@ static void build_schedule(kf_exec* E) {
   // periodic-fill needs: live-in rings whose box reaches beyond T on a periodic axis
   auto needs_fill = [&](const GroupExec& g, const Ver& v) {
     const Ring& R = g.L.rings[g.L.ring_of(v)];
-    for (int a = 0; a < 3; a++)   // (axes the kernel loads wrapped itself need no fill)
-      if (p.bc[a] == KF_BC_PERIODIC && !((g.L.wrap_axes >> a) & 1) && std::max(R.blo[a], R.bhi[a]) > 0) return true;
+    for (int a = 0; a < 3; a++)
+      if (p.bc[a] == KF_BC_PERIODIC && std::max(R.blo[a], R.bhi[a]) > 0) return true;
     return false;
   };
   std::set<int> all_fill;
@@ -1469,10 +1464,6 @@ kf_status kf_dist_create(kf_exec* const* parts, int32_t n_parts, int32_t px, int
                          const uint8_t* nccl_id, kf_dist** out) {
   KF_TRY({
     if (!out) fail(KF_E_ARG, "null argument");
-    for (int32_t i = 0; i < n_parts; i++)   // decomposed axes take their ghosts from the exchange
-      for (const GroupExec& g : parts[i]->G)
-        if ((px > 1 && (g.L.wrap_axes & 1)) || (py > 1 && (g.L.wrap_axes & 2)))
-          fail(KF_E_ARG, "a part was built with wrapload on an axis the decomposition splits (build it with wrapload = 0)");
     std::shared_ptr<Comm> comm;
     if (!(n_parts == px * py && world == 1)) {
       if (!nccl_id) fail(KF_E_ARG, "nccl_id required for the NCCL transport");

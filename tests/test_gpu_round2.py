@@ -180,50 +180,3 @@ def test_dist_graph_and_eager(graph):
     plan = kf.Program(desc).search(kf.SEARCH_HGGA, tgt, seed=1)[0]
     got = _loopback(desc, plan, inputs, 4, 2, 2, tgt, overlap=True, graph=graph)
     assert compare(desc, got, ref) == []
-
-
-@pytest.mark.parametrize("n,tile,pb", [((64, 48, 12), (32, 8, 0), (2, 1)),     # edge tiles on x and y
-                                       ((40, 36, 12), (32, 8, 0), (2, 1)),     # ragged x and y tiles
-                                       ((64, 48, 12), (64, 4, 0), (1, 1)),     # one tile spans x: both edges
-                                       ((40, 36, 12), (16, 4, 5), (1, 1))])    # z chunks, single points
-def test_wrapload_drops_fills(n, tile, pb):
-    """kf_target.wrapload: edge tiles load the wrapped parts of their boxes themselves (row bulk
-    copies from the opposite side, R9), no periodic ghost fill runs in the step, same results."""
-    desc = P.weather(n=n)
-    inputs = D.inputs_for(desc, 23)
-    ref = interp.run(desc, inputs, 3)
-    prog = kf.Program(desc)
-    tgt = kf.Target(tile=tile, pblock=pb, wrapload=1, minblocks=-1)
-    plan, _ = prog.search(kf.SEARCH_HGGA, tgt, seed=3)
-    got, ex = run_kf(desc, plan, inputs, 3, tgt)
-    assert ex.info().fills_per_step == 0
-    from .gpu_util import compare
-    assert compare(desc, got, ref) == [], (n, tile, pb)
-
-
-@pytest.mark.parametrize("dtype", [DT_F64, DT_F32])
-def test_wrapload_periodic_z_and_specials(dtype):
-    """Wrapped loads with a periodic z axis (planes wrap too) and x/y/z halos, on IEEE special
-    values, every legal plan."""
-    desc = special_program(dtype, bc=(BC_PERIODIC, BC_PERIODIC, BC_PERIODIC))
-    inputs = special_inputs(desc, 29)
-    ref = interp.run(desc, inputs, 2)
-    for plan in En.legal_plans(desc):
-        tgt = kf.Target(tile=(16, 4, 0), wrapload=1)
-        got, ex = run_kf(desc, plan, inputs, 2, tgt)
-        assert ex.info().fills_per_step == 0
-        assert compare_nan(desc, got, ref) == [], plan
-
-
-def test_wrapload_suite_fp32_every_plan():
-    """The test-suite program (fp32, stencils up to S27, periodic x/y) under wrapped loads."""
-    desc = P.gen_suite(seed=1, n=(40, 32, 12))
-    inputs = D.uniform(desc, 31)
-    ref = interp.run(desc, inputs, 2)
-    from .gpu_util import compare
-    tgt = kf.Target(tile=(32, 4, 0), wrapload=1)
-    plans = kf.Program(desc).legal_plans(tgt)
-    for plan in plans[:: max(1, len(plans) // 40)]:
-        got, ex = run_kf(desc, plan, inputs, 2, tgt)
-        assert ex.info().fills_per_step == 0
-        assert compare(desc, got, ref) == [], plan
