@@ -331,3 +331,32 @@ def test_plan_enumerate_equals_oracle_legal_set(which):
     ref = sorted(tuple(x) for x in En.legal_plans(desc))
     assert got == ref
     assert len(got) == p.count_legal()
+
+
+def test_hgga_at_scale_pinned_by_disjoint_union():
+    """NEXT-1 search pin at 49 kernels (where no exhaustive search of the whole program exists):
+    a program made of 7 independent Table V-style sub-programs (7 kernels each, no shared array,
+    kernels interleaved) has a known optimum -- legal groups cannot span two parts (V2 kinship),
+    bytes add over groups, so the optimum is the sum of the parts' optima, each by the ORACLE's
+    brute force (Bell(7) partitions).  The parts are ones where greedy merging is suboptimal, so
+    the pin separates the GA from the greedy baseline.  Every seed must reach the
+    optimum with a legal plan that is optimal part by part."""
+    from workloads.program import disjoint_union
+    seeds = [11, 12, 16, 20, 35, 46, 47]
+    parts = [P.gen_suite(n_kernels=7, n_arrays=6, seed=s, n=(64, 64, 32)) for s in seeds]
+    part_opt = [En.best_plan(q)[1] for q in parts]
+    desc, part_of = disjoint_union(parts, seed=2)
+    assert len(desc.kernels) == 49
+    p = kf.Program(desc)
+    _, greedy_b = p.search(kf.SEARCH_GREEDY)
+    assert greedy_b > sum(part_opt)                       # the instance is not greedy-easy
+    for seed in range(3):
+        plan, b = p.search(kf.SEARCH_HGGA_BYTES, seed=seed)
+        assert p.validate(plan)[0] == 0
+        assert b == sum(part_opt), (seed, b, sum(part_opt))
+        for i, q in enumerate(parts):                   # no group spans two parts; optimal per part
+            ks = [k for k in range(49) if part_of[k] == i]
+            assert not ({plan[k] for k in ks} & {plan[k] for k in range(49) if part_of[k] != i})
+            sub = [plan[k] for k in ks]
+            per, tb, _ = kf.Program(q).project(sub)
+            assert tb == part_opt[i]

@@ -215,3 +215,41 @@ def unroll(prog: Program, steps: int) -> Program:
     kernels = [Kernel(f"{k.name}@{s}", [Stmt(st.out, list(st.rpn)) for st in k.stmts])
                for s in range(steps) for k in prog.kernels]
     return prog.with_(name=prog.name if steps == 1 else f"{prog.name}x{steps}", kernels=kernels)
+
+
+def disjoint_union(parts: Sequence[Program], seed: int = 0) -> Tuple[Program, List[int]]:
+    """One program made of independent sub-programs: the arrays of every part renamed apart
+    (part index prefix), the kernels interleaved in a seeded random order that keeps each part's
+    own kernel order.  Returns the program and, per kernel, the part it came from.  Parts share
+    no array, so no dependence, sharing set or kinship chain crosses two parts: a legal group lies
+    inside one part and a plan of the union is a plan per part (the search pin at 40+ kernels).
+    All parts must have the same dtype, grid, ghost, boundary conditions and flags; PARAM slots
+    are re-indexed.  Pure description (no arithmetic of the method)."""
+    import numpy as np
+    p0 = parts[0]
+    for q in parts[1:]:
+        assert (q.dtype, tuple(q.n), tuple(q.ghost), tuple(q.bc), q.flags) == \
+            (p0.dtype, tuple(p0.n), tuple(p0.ghost), tuple(p0.bc), p0.flags)
+    arrays, params, aoff, poff = [], [], [], []
+    for i, q in enumerate(parts):
+        aoff.append(len(arrays))
+        poff.append(len(params))
+        arrays += [(f"p{i}_{nm}", fl) for nm, fl in q.arrays]
+        params += list(q.params)
+    queues = [list(range(len(q.kernels))) for q in parts]
+    order = [i for i, q in enumerate(parts) for _ in q.kernels]
+    np.random.default_rng(seed).shuffle(order)
+    kernels, part_of = [], []
+    for i in order:
+        k = parts[i].kernels[queues[i].pop(0)]
+
+        def mv(ins: Insn, i=i) -> Insn:
+            if ins.op == OP_LOAD:
+                return Insn(ins.op, ins.arg + aoff[i], ins.d, ins.imm)
+            if ins.op == OP_PARAM:
+                return Insn(ins.op, ins.arg + poff[i], ins.d, ins.imm)
+            return ins
+        kernels.append(Kernel(f"p{i}_{k.name}", [Stmt(st.out + aoff[i], [mv(x) for x in st.rpn]) for st in k.stmts]))
+        part_of.append(i)
+    return p0.with_(name="union_" + "_".join(q.name for q in parts), arrays=arrays, kernels=kernels,
+                    params=params), part_of
