@@ -417,7 +417,7 @@ def cpu_baseline(name: str, budget_s: float = 8.0):
 
 
 # ---------------------------------------------------------------- GPU timing
-AUTOTUNE_CANDIDATES = [  # (tile, stages, zunroll, ringunroll, minblocks, canvas_ld[, pblock x, pair_zq])
+AUTOTUNE_CANDIDATES = [  # (tile, stages, zunroll, ringunroll, minblocks, canvas_ld[, pblock x, pair_zq[, inline_xy]])
     ((32, 8, 64), 2, 1, 0, 0, 1), ((32, 8, 64), 2, 1, 0, -1, 1), ((32, 8, 64), 2, 1, 0, -1, 0), ((32, 8, 64), 2, 1, 0, 0, 0),
     ((32, 8, 32), 2, 1, 0, -1, 1), ((32, 8, 32), 2, 1, 0, 0, 0), ((32, 8, 0), 2, 1, 0, -1, 1), ((64, 4, 64), 2, 1, 0, 0, 1),
     ((32, 8, 64), 3, 1, 0, -1, 1), ((32, 8, 64), 2, 1, 1, -1, 1),
@@ -429,6 +429,8 @@ AUTOTUNE_CANDIDATES = [  # (tile, stages, zunroll, ringunroll, minblocks, canvas
     # z chunks of 43 planes: 3 chunks of a 128-plane column, 6.9 waves of 3 CTAs/SM instead of 4.6
     # (wave quantisation; measured -2..-4 % on the flux groups)
     ((32, 8, 43), 2, 1, 0, -1, 1, 2, 1), ((32, 8, 43), 2, 1, 0, -1, 1, 2, 0), ((32, 8, 43), 2, 1, 0, -1, 1),
+    # in-group values at xy offsets from shared memory instead of recomputed by their readers
+    ((32, 8, 43), 2, 1, 0, -1, 1, 2, 1, 0), ((32, 8, 32), 2, 1, 0, -1, 1, 2, 0, 0),
     # taller / wider pair tiles: less halo per point (36x20/512 = 1.41 vs 36x12/256 = 1.69 box/tile)
     ((32, 16, 43), 2, 1, 0, -1, 1, 2, 1), ((32, 16, 43), 2, 1, 0, -1, 1, 2, 0), ((64, 8, 43), 2, 1, 0, -1, 1, 2, 1),
     # three TMA stages for pairs: ncu showed 12 % of the flux group's warp samples waiting on the
@@ -442,15 +444,15 @@ def cand_kw(base_kw, c):
     kw = dict(base_kw)
     kw.update(tile=tuple(c[0]), stages=c[1], zunroll=c[2], ringunroll=c[3], minblocks=c[4] if len(c) > 4 else 0,
               canvas_ld=c[5] if len(c) > 5 else 1, pblock=(c[6] if len(c) > 6 else 1, 1),
-              pair_zq=c[7] if len(c) > 7 else 1)
+              pair_zq=c[7] if len(c) > 7 else 1, inline_xy=c[8] if len(c) > 8 else 1)
     return kw
 
 
 def cand_norm(c):
-    """Full 8-field form [tile, stages, zunroll, ringunroll, minblocks, canvas_ld, pblock_x, pair_zq]."""
-    full = list(c) + [None] * (8 - len(c))
-    dflt = [None, 2, 1, 0, 0, 1, 1, 1]
-    return [list(full[0])] + [full[i] if full[i] is not None else dflt[i] for i in range(1, 8)]
+    """Full 9-field form [tile, stages, zunroll, ringunroll, minblocks, canvas_ld, pblock_x, pair_zq, inline_xy]."""
+    full = list(c) + [None] * (9 - len(c))
+    dflt = [None, 2, 1, 0, 0, 1, 1, 1, 1]
+    return [list(full[0])] + [full[i] if full[i] is not None else dflt[i] for i in range(1, 9)]
 
 
 def autotune(prog, plan, dev, base_kw, steps=6):
@@ -975,7 +977,7 @@ def main():
     ap.add_argument("--no-parity", action="store_true")
     ap.add_argument("--autotune", type=int, default=1, help="per-group launch configuration by measurement (1/0)")
     ap.add_argument("--tuned", default=None, help="JSON per-group configs as printed in config.per_group_launch_config: "
-                                                  "[tile, stages, zunroll, ringunroll, minblocks, canvas_ld, pblock_x, pair_zq]")
+                                                  "[tile, stages, zunroll, ringunroll, minblocks, canvas_ld, pblock_x, pair_zq[, inline_xy]]")
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "kf":
         args.warmup = 3

@@ -187,8 +187,14 @@ typedef struct {
   int32_t pair_zq;               /* pair canvas (pblock 2x1): 1 = z-column values carried in
                                     registers across stream iterations instead of re-read
                                     from shared memory (more registers), 0 = off             */
+  int32_t inline_xy;             /* pair canvas: 1 = a reader recomputes an in-group value it reads
+                                    at an xy offset (the producer's statement re-evaluated there
+                                    from the staged inputs: same operations, same bits) instead
+                                    of a shared-memory copy behind a barrier, where the producer
+                                    reads only staged inputs and every reader runs in the same
+                                    stream iteration at dz = 0; 0 = shared-memory copies       */
 } kf_target;
-/* Fills the B200 defaults: 8.0e12, 232448, 255, 148, {64,4,0}, 2, 256, 16, 0, 1, {1,1}, 0, 0, 0, 0, 1, 1. */
+/* Fills the B200 defaults: 8.0e12, 232448, 255, 148, {64,4,0}, 2, 256, 16, 0, 1, {1,1}, 0, 0, 0, 0, 1, 1, 1. */
 kf_status kf_target_b200(kf_target* out);
 
 /* ------------------------------------------------------------------ legality (Eq. 1.1-1.7) */

@@ -65,7 +65,8 @@ class kf_target(C.Structure):
                 ("n_sm", C.c_int32), ("tile", C.c_int32 * 3), ("stages", C.c_int32), ("threads", C.c_int32),
                 ("max_halo", C.c_int32), ("internal_axes", C.c_int32), ("zunroll", C.c_int32),
                 ("pblock", C.c_int32 * 2), ("ringunroll", C.c_int32), ("ghostwrite", C.c_int32),
-                ("minblocks", C.c_int32), ("skew", C.c_int32), ("canvas_ld", C.c_int32), ("pair_zq", C.c_int32)]
+                ("minblocks", C.c_int32), ("skew", C.c_int32), ("canvas_ld", C.c_int32), ("pair_zq", C.c_int32),
+                ("inline_xy", C.c_int32)]
 
 
 class kf_violation(C.Structure):

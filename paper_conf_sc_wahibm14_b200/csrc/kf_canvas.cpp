@@ -66,7 +66,40 @@ CanvasPlan plan_canvas(const Program& p, const GroupLowering& L) {
     c.rounds = (c.cwp * c.ch + L.threads - 1) / L.threads;
     c.pair = c.ok = c.rounds == 1;
   }
-  // versions whose every in-group read is forwarded need no shared-memory copy in fast iterations
+  // Inline recompute (pair mode, L.inline_xy): an in-group version whose statement reads only
+  // staged live-in versions, and whose every in-group reader runs in the same stream iteration
+  // (equal delay) and reads it in its own plane (dz = 0), is recomputed by each reader at each xy
+  // offset it reads (the same IEEE operations in the same order: the same bits) instead of being
+  // stored to and re-read from shared memory behind a barrier.  The loads this adds lie in the
+  // live-in boxes (a box covers the producer's region grown by its footprint, and the producer's
+  // region covers its readers' regions grown by theirs).  Fast iterations only: the slow path
+  // keeps the ring (same-iteration readers: its contents never cross iterations).
+  if (c.pair && L.inline_xy)
+    for (int k : alive) {
+      const Kernel& K = p.kernels[k];
+      for (size_t si = 0; si < K.stmts.size(); si++) {
+        const Ver V{K.stmts[si].out, p.vw(k, K.stmts[si].out)};
+        if (L.ring_of(V) < 0) continue;
+        bool ok = true, any_xy = false;
+        for (const Insn& in : K.stmts[si].rpn)
+          if (in.op == KF_OP_LOAD) {
+            const int r = L.ring_of(Ver{in.arg, p.vr(k, in.arg)});
+            if (r < 0 || !L.rings[r].live_in) ok = false;
+          }
+        for (int c2 : alive) {
+          auto it = p.kernels[c2].reads.find(V.x);
+          if (c2 == k || it == p.kernels[c2].reads.end() || p.vr(c2, V.x) != V.v) continue;
+          if (L.delay.at(c2) != L.delay.at(k)) ok = false;
+          for (auto& d : it->second) {
+            if (d[2] != 0) ok = false;
+            if (d[0] != 0 || d[1] != 0) any_xy = true;
+          }
+        }
+        if (ok && any_xy) c.inl[V] = {k, int(si)};
+      }
+    }
+  // versions whose every in-group read is forwarded (or recomputed) need no shared-memory copy in
+  // fast iterations
   for (int k : alive)
     for (auto& [x, offs] : p.kernels[k].reads) {
       const int v = p.vr(k, x);
@@ -74,7 +107,7 @@ CanvasPlan plan_canvas(const Program& p, const GroupLowering& L) {
       for (auto& d : offs)
         for (int uu = 0; uu < U; uu++) {
           int pr, u2;
-          if (!canvas_forward(p, L, k, x, d, uu, &pr, &u2)) c.need_sts.insert(Ver{x, v});
+          if (!canvas_forward(p, L, k, x, d, uu, &pr, &u2) && !c.inlined(p, k, x, d)) c.need_sts.insert(Ver{x, v});
         }
     }
   // phases: a barrier only before a kernel that reads through shared memory a plane written (to
@@ -92,7 +125,7 @@ CanvasPlan plan_canvas(const Program& p, const GroupLowering& L) {
         for (auto& d : offs)
           for (int uu = 0; uu < U; uu++) {
             int q, u2;
-            if (canvas_forward(p, L, k, x, d, uu, &q, &u2)) continue;
+            if (canvas_forward(p, L, k, x, d, uu, &q, &u2) || c.inlined(p, k, x, d)) continue;
             if (L.delay.at(k) - d[2] - L.delay.at(pr) < U) need = true;
           }
       }
@@ -114,13 +147,22 @@ CanvasPlan plan_canvas(const Program& p, const GroupLowering& L) {
         for (int uu = 0; uu < U; uu++) {
           int pr, u2;
           if (canvas_forward(p, L, k, x, d, uu, &pr, &u2)) continue;
-          const CanvasKey key = canvas_key(p, L, c, k, x, d, uu);
-          auto it = c.krect.find(key);
-          if (it == c.krect.end()) c.krect[key] = rk;
-          else {
-            auto& a = it->second;
-            a = {std::min(a[0], rk[0]), std::max(a[1], rk[1]), std::min(a[2], rk[2]), std::max(a[3], rk[3])};
+          auto add = [&](int kr, int xr, const Off& dr) {
+            const CanvasKey key = canvas_key(p, L, c, kr, xr, dr, uu);
+            auto it = c.krect.find(key);
+            if (it == c.krect.end()) c.krect[key] = rk;
+            else {
+              auto& a = it->second;
+              a = {std::min(a[0], rk[0]), std::max(a[1], rk[1]), std::min(a[2], rk[2]), std::max(a[3], rk[3])};
+            }
+          };
+          if (c.inlined(p, k, x, d)) {   // the producer's loads, shifted by the read's offset
+            const auto& [pk, si] = c.inl.at(Ver{x, p.vr(k, x)});
+            for (const Insn& in : p.kernels[pk].stmts[si].rpn)
+              if (in.op == KF_OP_LOAD) add(pk, in.arg, Off{d[0] + in.d[0], d[1] + in.d[1], d[2] + in.d[2]});
+            continue;
           }
+          add(k, x, d);
         }
   }
   // shared-memory traffic of one fast iteration (U planes of one tile)

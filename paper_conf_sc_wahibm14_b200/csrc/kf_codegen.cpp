@@ -649,23 +649,39 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
   // and the z-flux read at dz = -1); after a slow iteration they are reloaded once.
   struct PSrc { bool is_load; PK src; int x, v; };
   std::map<PK, PSrc> pcarry;
+  // The reads a kernel issues for its point j of the pair: its own loads, a read of an inlined
+  // version at an xy offset replaced by the producer's loads shifted by that offset -- none where
+  // the offset lands on the thread's other point (the producer's value there is forwarded).
+  auto eff_reads = [&](int k, int j, const std::function<void(int, int, const Off&)>& fn) {
+    for (auto& [x, offs] : p.kernels[k].reads)
+      for (auto& d : offs) {
+        if (cv.inlined(p, k, x, d)) {
+          const int ax = j + d[0];
+          if (d[1] == 0 && (ax == 0 || ax == 1)) continue;
+          const auto& [pk, si] = cv.inl.at(Ver{x, p.vr(k, x)});
+          for (const Insn& in : p.kernels[pk].stmts[si].rpn)
+            if (in.op == KF_OP_LOAD) fn(pk, in.arg, Off{d[0] + in.d[0], d[1] + in.d[1], d[2] + in.d[2]});
+          continue;
+        }
+        fn(k, x, d);
+      }
+  };
   if (pair_mode) {
     for (int k : alive)
-      for (auto& [x, offs] : p.kernels[k].reads)
-        for (auto& d : offs)
-          for (int j = 0; j < 2; j++) {
-            int pr, u2, comp;
-            if (fwd_src(k, x, d, 0, &pr, &u2)) continue;
-            const Rect rc = krect.at(load_key(k, x, d, 0));
-            const PK pk = pk_of(k, x, d, j, &comp);
-            const Rect rj{rc[0] - j, rc[1] - j, rc[2], rc[3]};
-            auto it = pall.find(pk);
-            if (it == pall.end()) pall[pk] = rj;
-            else {
-              auto& a = it->second;
-              a = {std::min(a[0], rj[0]), std::max(a[1], rj[1]), std::min(a[2], rj[2]), std::max(a[3], rj[3])};
-            }
+      for (int j = 0; j < 2; j++)
+        eff_reads(k, j, [&](int kr, int x, const Off& d) {
+          int pr, u2, comp;
+          if (fwd_src(kr, x, d, 0, &pr, &u2)) return;
+          const Rect rc = krect.at(load_key(kr, x, d, 0));
+          const PK pk = pk_of(kr, x, d, j, &comp);
+          const Rect rj{rc[0] - j, rc[1] - j, rc[2], rc[3]};
+          auto it = pall.find(pk);
+          if (it == pall.end()) pall[pk] = rj;
+          else {
+            auto& a = it->second;
+            a = {std::min(a[0], rj[0]), std::max(a[1], rj[1]), std::min(a[2], rj[2]), std::max(a[3], rj[3])};
           }
+        });
     if (L.pair_zq)
       for (auto& [pk, rc] : pall) {   // ascending (ring, plane offset): widening propagates upward
         const auto& [ring, po, rel] = pk;
@@ -727,7 +743,89 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
     std::map<PK, Rect> prect;
     std::map<PK, int> pmask;   // elements of the pair needed (bit 0: first, bit 1: second)
     std::map<PK, std::string> ldname;
+    size_t cur_ph = 0;
+    // the value a reader's LOAD takes for point j: forwarded, carried, or a (CSE'd) shared load
+    auto load_val = [&](int kr, int x, const Off& d, int j) -> std::string {
+      int pr, u2, comp;
+      if (fwd_src(kr, x, d, 0, &pr, &u2)) return fwd.at(std::make_tuple(x, p.vr(kr, x), j));
+      const PK pk = pk_of(kr, x, d, j, &comp);
+      if (pcarry.count(pk)) return pq_name(pk) + (comp ? ".y" : ".x");
+      auto it = ldname.find(pk);
+      if (it == ldname.end()) {
+        const auto& [ring, po, rel] = pk;
+        const Rect& rc = pall.at(pk);   // (widened for z-queue carries)
+        const std::string nm = "pl" + std::to_string(ring) + "_" + (po < 0 ? "m" + std::to_string(-po) : std::to_string(po)) +
+                               "_" + (rel < 0 ? "m" + std::to_string(-rel) : std::to_string(rel)) + "_h" + std::to_string(cur_ph);
+        const int mask = pmask.at(pk);
+        if (mask == 3) {
+          if (pair_nopred(pk))
+            o << "      const real2 " << nm << " = " << pair_acc(pk) << ";\n";
+          else
+            o << "      const real2 " << nm << " = (" << pair_pred(rc) << ") ? " << pair_acc(pk)
+              << " : real2{(real)0, (real)0};\n";
+        } else {
+          const int c1 = mask == 2 ? 1 : 0;
+          const std::string b1 = L.canvas_ld ? cbase(pall.at(pk), L.rings[ring].px)
+                                             : "cb" + std::to_string(L.rings[ring].px) + "_r0";
+          const std::string acc1 = "P" + std::to_string(ring) + "_" + std::to_string(slot(ring, po)) + "[" + b1 + " + " +
+                                   std::to_string(rel + c1) + "]";
+          if (pair_nopred(pk)) o << "      const real " << nm << " = " << acc1 << ";\n";
+          else o << "      const real " << nm << " = (" << pair_pred(rc) << ") ? " << acc1 << " : (real)0;\n";
+        }
+        it = ldname.emplace(pk, nm).first;
+        ldfirst_p.emplace(pk, nm);
+      }
+      return it->second + (pmask.at(pk) == 3 ? (comp ? ".y" : ".x") : "");
+    };
+    // an inlined version at xy offset d of point j: the producer's statement re-evaluated there
+    // (same operations, same order), once per (statement, point) per iteration
+    std::map<std::tuple<int, int, int, int>, std::string> inl_memo;
+    auto inline_val = [&](int k, int x, const Off& d, int j) -> std::string {
+      const auto [pk, si] = cv.inl.at(Ver{x, p.vr(k, x)});
+      const int ax = j + d[0];
+      if (d[1] == 0 && (ax == 0 || ax == 1)) return fwd.at(std::make_tuple(x, p.vr(k, x), ax));
+      const auto mk = std::make_tuple(pk, si, ax, d[1]);
+      auto mit = inl_memo.find(mk);
+      if (mit != inl_memo.end()) return mit->second;
+      auto sg = [](int v) { return v < 0 ? "m" + std::to_string(-v) : std::to_string(v); };
+      const std::string pre = "n" + std::to_string(pk) + "s" + std::to_string(si) + "_" + sg(ax) + "_" + sg(d[1]) + "_";
+      std::vector<std::string> st;
+      int tmp = 0;
+      for (const Insn& in : p.kernels[pk].stmts[si].rpn) {
+        std::string f;
+        switch (in.op) {
+          case KF_OP_CONST: f = lit(in.imm, p.dtype); break;
+          case KF_OP_PARAM: f = "(real)a.prm[" + std::to_string(in.arg) + "]"; break;
+          case KF_OP_LOAD: f = load_val(pk, in.arg, Off{d[0] + in.d[0], d[1] + in.d[1], d[2] + in.d[2]}, j); break;
+          case KF_OP_NEG: case KF_OP_ABS: case KF_OP_SQRT: {
+            std::string a1 = st.back(); st.pop_back();
+            f = in.op == KF_OP_NEG ? "-" + a1
+              : in.op == KF_OP_ABS ? (p.dtype == KF_F32 ? "fabsf(" : "fabs(") + a1 + ")"
+                                   : (p.dtype == KF_F32 ? "sqrtf(" : "sqrt(") + a1 + ")";
+            break;
+          }
+          default: {
+            std::string b = st.back(); st.pop_back();
+            std::string a1 = st.back(); st.pop_back();
+            switch (in.op) {
+              case KF_OP_ADD: f = a1 + " + " + b; break;
+              case KF_OP_SUB: f = a1 + " - " + b; break;
+              case KF_OP_MUL: f = a1 + " * " + b; break;
+              case KF_OP_DIV: f = a1 + " / " + b; break;
+              case KF_OP_MIN: f = "(" + b + " < " + a1 + ") ? " + b + " : " + a1; break;
+              case KF_OP_MAX: f = "(" + a1 + " < " + b + ") ? " + b + " : " + a1; break;
+            }
+          }
+        }
+        const std::string t = pre + std::to_string(tmp++);
+        o << "      const real " << t << " = " << f << ";\n";
+        st.push_back(t);
+      }
+      inl_memo.emplace(mk, st.back());
+      return st.back();
+    };
     for (size_t ph = 0; ph < cph.size(); ph++) {
+      cur_ph = ph;
       if (ph > 0) o << "      __syncthreads();\n";
       // lanes (first point's canvas x, row) needing each pair load in this phase (all phases
       // unless per-phase loads)
@@ -737,22 +835,21 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
         ldname.clear();
       }
       for (int k : (phase_ld ? cph[ph] : ph == 0 ? alive : std::vector<int>{}))
-        for (auto& [x, offs] : p.kernels[k].reads)
-          for (auto& d : offs)
-            for (int j = 0; j < 2; j++) {
-              int pr, u2, comp;
-              if (fwd_src(k, x, d, 0, &pr, &u2)) continue;
-              const Rect rc = krect.at(load_key(k, x, d, 0));
-              const PK pk = pk_of(k, x, d, j, &comp);
-              const Rect rj{rc[0] - j, rc[1] - j, rc[2], rc[3]};
-              pmask[pk] |= 1 << comp;
-              auto it = prect.find(pk);
-              if (it == prect.end()) prect[pk] = rj;
-              else {
-                auto& a = it->second;
-                a = {std::min(a[0], rj[0]), std::max(a[1], rj[1]), std::min(a[2], rj[2]), std::max(a[3], rj[3])};
-              }
+        for (int j = 0; j < 2; j++)
+          eff_reads(k, j, [&](int kr, int x, const Off& d) {
+            int pr, u2, comp;
+            if (fwd_src(kr, x, d, 0, &pr, &u2)) return;
+            const Rect rc = krect.at(load_key(kr, x, d, 0));
+            const PK pk = pk_of(kr, x, d, j, &comp);
+            const Rect rj{rc[0] - j, rc[1] - j, rc[2], rc[3]};
+            pmask[pk] |= 1 << comp;
+            auto it = prect.find(pk);
+            if (it == prect.end()) prect[pk] = rj;
+            else {
+              auto& a = it->second;
+              a = {std::min(a[0], rj[0]), std::max(a[1], rj[1]), std::min(a[2], rj[2]), std::max(a[3], rj[3])};
             }
+          });
       // a pair of which only one element is needed (e.g. y/z neighbours in a ring whose pairs are
       // offset by one from the canvas pairs) is a scalar load: same instruction count as the
       // vector load, half the wavefronts; carry sources and carried values stay vectors
@@ -775,45 +872,9 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
               switch (in.op) {
                 case KF_OP_CONST: f = lit(in.imm, p.dtype); break;
                 case KF_OP_PARAM: f = "(real)a.prm[" + std::to_string(in.arg) + "]"; break;
-                case KF_OP_LOAD: {
-                  int pr, u2, comp;
-                  if (fwd_src(k, in.arg, in.d, 0, &pr, &u2)) {
-                    f = fwd.at(std::make_tuple(in.arg, p.vr(k, in.arg), j));
-                    break;
-                  }
-                  const PK pk = pk_of(k, in.arg, in.d, j, &comp);
-                  if (pcarry.count(pk)) {
-                    f = pq_name(pk) + (comp ? ".y" : ".x");
-                    break;
-                  }
-                  auto it = ldname.find(pk);
-                  if (it == ldname.end()) {
-                    const auto& [ring, po, rel] = pk;
-                    const Rect& rc = pall.at(pk);   // (widened for z-queue carries)
-                    const std::string nm = "pl" + std::to_string(ring) + "_" + (po < 0 ? "m" + std::to_string(-po) : std::to_string(po)) +
-                                           "_" + (rel < 0 ? "m" + std::to_string(-rel) : std::to_string(rel)) + "_h" + std::to_string(ph);
-                    const int mask = pmask.at(pk);
-                    if (mask == 3) {
-                      if (pair_nopred(pk))
-                        o << "      const real2 " << nm << " = " << pair_acc(pk) << ";\n";
-                      else
-                        o << "      const real2 " << nm << " = (" << pair_pred(rc) << ") ? " << pair_acc(pk)
-                          << " : real2{(real)0, (real)0};\n";
-                    } else {
-                      const int c1 = mask == 2 ? 1 : 0;
-                      const std::string b1 = L.canvas_ld ? cbase(pall.at(pk), L.rings[ring].px)
-                                                         : "cb" + std::to_string(L.rings[ring].px) + "_r0";
-                      const std::string acc1 = "P" + std::to_string(ring) + "_" + std::to_string(slot(ring, po)) + "[" + b1 + " + " +
-                                               std::to_string(rel + c1) + "]";
-                      if (pair_nopred(pk)) o << "      const real " << nm << " = " << acc1 << ";\n";
-                      else o << "      const real " << nm << " = (" << pair_pred(rc) << ") ? " << acc1 << " : (real)0;\n";
-                    }
-                    it = ldname.emplace(pk, nm).first;
-                    ldfirst_p.emplace(pk, nm);
-                  }
-                  f = it->second + (pmask.at(pk) == 3 ? (comp ? ".y" : ".x") : "");
+                case KF_OP_LOAD:
+                  f = cv.inlined(p, k, in.arg, in.d) ? inline_val(k, in.arg, in.d, j) : load_val(k, in.arg, in.d, j);
                   break;
-                }
                 case KF_OP_NEG: case KF_OP_ABS: case KF_OP_SQRT: {
                   std::string a1 = st.back(); st.pop_back();
                   f = in.op == KF_OP_NEG ? "-" + a1

@@ -135,6 +135,7 @@ struct GroupLowering {
   int ring_unroll = 0;      // 0, or N: every ring size a power of two dividing N, loop unrolled N times
   bool ghost_write = false; // live-out stores also write the periodic x/y ghost copies (no fills)
   int pair_zq = 1;          // pair canvas: z-column register queues (kf_target.pair_zq)
+  int inline_xy = 0;        // pair canvas: readers recompute in-group versions at xy offsets
   int canvas_ld = 1;        // fast-iteration shared loads unpredicated where in bounds (kf_target.canvas_ld)
   int minblocks = 0;        // __launch_bounds__ min CTAs/SM: 0 auto (SMEM-limited), -1 none, n
   int ring_of(const Ver& v) const;        // index in rings or -1
@@ -186,6 +187,12 @@ struct CanvasPlan {
   // an even (16-byte for fp64) element; shared loads/stores and live-out stores are 2-wide vectors
   bool pair = false;
   int lop = 0, hip = 0, cwp = 0;   // pair columns left of / right of the tile, per canvas row
+  // pair mode with L.inline_xy: in-group versions whose readers recompute them at their xy
+  // offsets instead of reading a shared-memory copy: version -> (producer, statement index)
+  std::map<Ver, std::pair<int, int>> inl;
+  bool inlined(const Program& p, int k, int x, const Off& d) const {
+    return (d[0] != 0 || d[1] != 0) && inl.count(Ver{x, p.vr(k, x)}) > 0;
+  }
 };
 bool canvas_forward(const Program& p, const GroupLowering& L, int k, int x, const Off& d, int uu, int* prod, int* up);
 CanvasKey canvas_key(const Program& p, const GroupLowering& L, const CanvasPlan& c, int k, int x, const Off& d, int uu);

@@ -358,6 +358,7 @@ kf_status kf_target_b200(kf_target* out) {
     t.skew = 0;
     t.canvas_ld = 1;
     t.pair_zq = 1;
+    t.inline_xy = 1;   // measured: -1.6 % step, flux groups -2 .. -6 % (profiles/round2_summary.md)
     *out = t;
   });
 }

@@ -29,8 +29,8 @@ def test_workloads_weak_and_strong_grids():
 
 
 def test_candidate_normal_form():
-    assert bench.cand_norm(((32, 8, 64), 2, 1, 0, 0, 1)) == [[32, 8, 64], 2, 1, 0, 0, 1, 1, 1]
-    assert bench.cand_norm(((32, 8, 43), 3, 1, 0, -1, 1, 2, 0)) == [[32, 8, 43], 3, 1, 0, -1, 1, 2, 0]
+    assert bench.cand_norm(((32, 8, 64), 2, 1, 0, 0, 1)) == [[32, 8, 64], 2, 1, 0, 0, 1, 1, 1, 1]
+    assert bench.cand_norm(((32, 8, 43), 3, 1, 0, -1, 1, 2, 0)) == [[32, 8, 43], 3, 1, 0, -1, 1, 2, 0, 1]
     kw = bench.cand_kw({"tile": (32, 8, 64)}, [[64, 4, 64], 2, 2, 1, -1, 0, 2, 0])
     assert kw["tile"] == (64, 4, 64) and kw["zunroll"] == 2 and kw["pblock"] == (2, 1) and kw["canvas_ld"] == 0
 
