@@ -192,7 +192,9 @@ typedef struct {
                                     from the staged inputs: same operations, same bits) instead
                                     of a shared-memory copy behind a barrier, where the producer
                                     reads only staged inputs and every reader runs in the same
-                                    stream iteration at dz = 0; 0 = shared-memory copies       */
+                                    stream iteration at dz = 0; 2 = also producers reading such
+                                    recomputed values (two levels: more recompute, registers);
+                                    0 = shared-memory copies                                  */
 } kf_target;
 /* Fills the B200 defaults: 8.0e12, 232448, 255, 148, {64,4,0}, 2, 256, 16, 0, 1, {1,1}, 0, 0, 0, 0, 1, 1, 1. */
 kf_status kf_target_b200(kf_target* out);

@@ -4,6 +4,7 @@
 // and by the resource-aware projection (model_time), so the model counts the shared-memory
 // traffic the generated kernel actually issues.
 #include <algorithm>
+#include <functional>
 
 #include "kf_internal.hpp"
 
@@ -75,28 +76,35 @@ CanvasPlan plan_canvas(const Program& p, const GroupLowering& L) {
   // region covers its readers' regions grown by theirs).  Fast iterations only: the slow path
   // keeps the ring (same-iteration readers: its contents never cross iterations).
   if (c.pair && L.inline_xy)
-    for (int k : alive) {
-      const Kernel& K = p.kernels[k];
-      for (size_t si = 0; si < K.stmts.size(); si++) {
-        const Ver V{K.stmts[si].out, p.vw(k, K.stmts[si].out)};
-        if (L.ring_of(V) < 0) continue;
-        bool ok = true, any_xy = false;
-        for (const Insn& in : K.stmts[si].rpn)
-          if (in.op == KF_OP_LOAD) {
-            const int r = L.ring_of(Ver{in.arg, p.vr(k, in.arg)});
-            if (r < 0 || !L.rings[r].live_in) ok = false;
+    for (int level = 0; level < (L.inline_xy >= 2 ? 2 : 1); level++) {   // level 1 (inline_xy 2): statements that also read level-0 values
+      std::map<Ver, std::pair<int, int>> add;
+      for (int k : alive) {
+        const Kernel& K = p.kernels[k];
+        for (size_t si = 0; si < K.stmts.size(); si++) {
+          const Ver V{K.stmts[si].out, p.vw(k, K.stmts[si].out)};
+          if (L.ring_of(V) < 0 || c.inl.count(V)) continue;
+          bool ok = true, any_xy = false;
+          for (const Insn& in : K.stmts[si].rpn)
+            if (in.op == KF_OP_LOAD) {
+              const Ver W{in.arg, p.vr(k, in.arg)};
+              const int r = L.ring_of(W);
+              if (r < 0 || !(L.rings[r].live_in || c.inl.count(W))) ok = false;
+            }
+          for (int c2 : alive) {
+            auto it = p.kernels[c2].reads.find(V.x);
+            if (c2 == k || it == p.kernels[c2].reads.end() || p.vr(c2, V.x) != V.v) continue;
+            if (L.delay.at(c2) != L.delay.at(k)) ok = false;
+            for (auto& d : it->second) {
+              if (d[2] != 0) ok = false;
+              if (d[0] != 0 || d[1] != 0) any_xy = true;
+            }
           }
-        for (int c2 : alive) {
-          auto it = p.kernels[c2].reads.find(V.x);
-          if (c2 == k || it == p.kernels[c2].reads.end() || p.vr(c2, V.x) != V.v) continue;
-          if (L.delay.at(c2) != L.delay.at(k)) ok = false;
-          for (auto& d : it->second) {
-            if (d[2] != 0) ok = false;
-            if (d[0] != 0 || d[1] != 0) any_xy = true;
-          }
+          (void)any_xy;   // (values read only at offset 0 join too: the inputs of level-1 values)
+          if (ok) add[V] = {k, int(si)};
         }
-        if (ok && any_xy) c.inl[V] = {k, int(si)};
       }
+      if (add.empty()) break;
+      c.inl.insert(add.begin(), add.end());
     }
   // versions whose every in-group read is forwarded (or recomputed) need no shared-memory copy in
   // fast iterations
@@ -156,13 +164,18 @@ CanvasPlan plan_canvas(const Program& p, const GroupLowering& L) {
               a = {std::min(a[0], rk[0]), std::max(a[1], rk[1]), std::min(a[2], rk[2]), std::max(a[3], rk[3])};
             }
           };
-          if (c.inlined(p, k, x, d)) {   // the producer's loads, shifted by the read's offset
-            const auto& [pk, si] = c.inl.at(Ver{x, p.vr(k, x)});
-            for (const Insn& in : p.kernels[pk].stmts[si].rpn)
-              if (in.op == KF_OP_LOAD) add(pk, in.arg, Off{d[0] + in.d[0], d[1] + in.d[1], d[2] + in.d[2]});
-            continue;
-          }
-          add(k, x, d);
+          // an inlined read: the producer's loads shifted by the read's offset, recursively
+          std::function<void(int, int, const Off&)> expand = [&](int kr, int xr, const Off& dr) {
+            int q, u3;
+            if (c.inlined(p, kr, xr, dr)) {
+              const auto& [pk, si] = c.inl.at(Ver{xr, p.vr(kr, xr)});
+              for (const Insn& in : p.kernels[pk].stmts[si].rpn)
+                if (in.op == KF_OP_LOAD) expand(pk, in.arg, Off{dr[0] + in.d[0], dr[1] + in.d[1], dr[2] + in.d[2]});
+            } else if (!canvas_forward(p, L, kr, xr, dr, uu, &q, &u3)) {
+              add(kr, xr, dr);
+            }
+          };
+          expand(k, x, d);
         }
   }
   // shared-memory traffic of one fast iteration (U planes of one tile)

@@ -652,19 +652,22 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
   // The reads a kernel issues for its point j of the pair: its own loads, a read of an inlined
   // version at an xy offset replaced by the producer's loads shifted by that offset -- none where
   // the offset lands on the thread's other point (the producer's value there is forwarded).
+  // (recursively: an inlined producer may itself read inlined values, R20d)
+  std::function<void(int, int, const Off&, int, const std::function<void(int, int, const Off&)>&)> eff_expand =
+      [&](int kr, int x, const Off& d, int j, const std::function<void(int, int, const Off&)>& fn) {
+        if (cv.inlined(p, kr, x, d)) {
+          const int ax = j + d[0];
+          if (d[1] == 0 && (ax == 0 || ax == 1)) return;
+          const auto& [pk, si] = cv.inl.at(Ver{x, p.vr(kr, x)});
+          for (const Insn& in : p.kernels[pk].stmts[si].rpn)
+            if (in.op == KF_OP_LOAD) eff_expand(pk, in.arg, Off{d[0] + in.d[0], d[1] + in.d[1], d[2] + in.d[2]}, j, fn);
+          return;
+        }
+        fn(kr, x, d);
+      };
   auto eff_reads = [&](int k, int j, const std::function<void(int, int, const Off&)>& fn) {
     for (auto& [x, offs] : p.kernels[k].reads)
-      for (auto& d : offs) {
-        if (cv.inlined(p, k, x, d)) {
-          const int ax = j + d[0];
-          if (d[1] == 0 && (ax == 0 || ax == 1)) continue;
-          const auto& [pk, si] = cv.inl.at(Ver{x, p.vr(k, x)});
-          for (const Insn& in : p.kernels[pk].stmts[si].rpn)
-            if (in.op == KF_OP_LOAD) fn(pk, in.arg, Off{d[0] + in.d[0], d[1] + in.d[1], d[2] + in.d[2]});
-          continue;
-        }
-        fn(k, x, d);
-      }
+      for (auto& d : offs) eff_expand(k, x, d, j, fn);
   };
   if (pair_mode) {
     for (int k : alive)
@@ -780,7 +783,7 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
     // an inlined version at xy offset d of point j: the producer's statement re-evaluated there
     // (same operations, same order), once per (statement, point) per iteration
     std::map<std::tuple<int, int, int, int>, std::string> inl_memo;
-    auto inline_val = [&](int k, int x, const Off& d, int j) -> std::string {
+    std::function<std::string(int, int, const Off&, int)> inline_val = [&](int k, int x, const Off& d, int j) -> std::string {
       const auto [pk, si] = cv.inl.at(Ver{x, p.vr(k, x)});
       const int ax = j + d[0];
       if (d[1] == 0 && (ax == 0 || ax == 1)) return fwd.at(std::make_tuple(x, p.vr(k, x), ax));
@@ -796,7 +799,11 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
         switch (in.op) {
           case KF_OP_CONST: f = lit(in.imm, p.dtype); break;
           case KF_OP_PARAM: f = "(real)a.prm[" + std::to_string(in.arg) + "]"; break;
-          case KF_OP_LOAD: f = load_val(pk, in.arg, Off{d[0] + in.d[0], d[1] + in.d[1], d[2] + in.d[2]}, j); break;
+          case KF_OP_LOAD: {
+            const Off dd{d[0] + in.d[0], d[1] + in.d[1], d[2] + in.d[2]};
+            f = cv.inlined(p, pk, in.arg, dd) ? inline_val(pk, in.arg, dd, j) : load_val(pk, in.arg, dd, j);
+            break;
+          }
           case KF_OP_NEG: case KF_OP_ABS: case KF_OP_SQRT: {
             std::string a1 = st.back(); st.pop_back();
             f = in.op == KF_OP_NEG ? "-" + a1

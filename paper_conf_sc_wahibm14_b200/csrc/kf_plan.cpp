@@ -85,7 +85,7 @@ GroupLowering lower_group(const Program& p, const std::vector<int>& g, const kf_
   L.canvas_ld = t.canvas_ld;
   L.pair_zq = t.pair_zq;
   L.inline_xy = t.inline_xy;
-  if (const char* v = getenv("KF_INLINE")) L.inline_xy = atoi(v) ? 1 : 0;   // A/B switch
+  if (const char* v = getenv("KF_INLINE")) L.inline_xy = std::min(2, std::max(0, atoi(v)));   // A/B switch
   L.pblock[0] = t.pblock[0];
   L.pblock[1] = t.pblock[1];
   L.live_in = group_live_in(p, g);
@@ -572,7 +572,7 @@ void check_target(const kf_target* t) {
   if (t->skew < 0 || t->skew > 1) fail(KF_E_ARG, "skew must be 0 or 1");
   if (t->canvas_ld < 0 || t->canvas_ld > 1) fail(KF_E_ARG, "canvas_ld must be 0 or 1");
   if (t->pair_zq < 0 || t->pair_zq > 1) fail(KF_E_ARG, "pair_zq must be 0 or 1");
-  if (t->inline_xy < 0 || t->inline_xy > 1) fail(KF_E_ARG, "inline_xy must be 0 or 1");
+  if (t->inline_xy < 0 || t->inline_xy > 2) fail(KF_E_ARG, "inline_xy must be 0, 1 or 2");
   if (t->pblock[0] < 1 || t->pblock[0] > 4 || t->pblock[1] < 1 || t->pblock[1] > 4)
     fail(KF_E_ARG, "pblock must be in [1, 4] x [1, 4]");
   if (t->threads < 32 || t->threads > 1024 || t->threads % 32) fail(KF_E_ARG, "threads must be a multiple of 32 in [32,1024]");

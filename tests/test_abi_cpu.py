@@ -248,7 +248,7 @@ def test_target_knobs_validated():
     desc = P.tiny()
     p = kf.Program(desc)
     for bad in (dict(canvas_ld=2), dict(pair_zq=-1), dict(skew=2), dict(minblocks=-2), dict(pblock=(5, 1)),
-                dict(tile=(30, 8, 0)), dict(inline_xy=2)):
+                dict(tile=(30, 8, 0)), dict(inline_xy=3)):
         with pytest.raises(kf.KfError):
             p.project([0, 0, 1], kf.Target(**bad))
 
@@ -264,7 +264,8 @@ def test_codegen_pair_canvas_and_split_compile_for_sm100a():
     checked = 0
     for seed in (1, 2):
         plan, _ = p.search(kf.SEARCH_HGGA, t, seed=seed)
-        for kw in (dict(pblock=(2, 1)), dict(pblock=(2, 1), canvas_ld=0, pair_zq=0), dict(), dict(pblock=(2, 1), inline_xy=0)):
+        for kw in (dict(pblock=(2, 1)), dict(pblock=(2, 1), canvas_ld=0, pair_zq=0), dict(), dict(pblock=(2, 1), inline_xy=0),
+                   dict(pblock=(2, 1), inline_xy=2)):
             tt = kf.Target(tile=(32, 8, 0), **kw)
             per, _, _ = p.project(plan, tt)
             for g in range(max(plan) + 1):

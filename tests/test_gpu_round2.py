@@ -180,3 +180,32 @@ def test_dist_graph_and_eager(graph):
     plan = kf.Program(desc).search(kf.SEARCH_HGGA, tgt, seed=1)[0]
     got = _loopback(desc, plan, inputs, 4, 2, 2, tgt, overlap=True, graph=graph)
     assert compare(desc, got, ref) == []
+
+
+@pytest.mark.parametrize("level", [0, 1, 2])
+def test_inline_recompute_levels_bit_exact(level):
+    """kf_target.inline_xy (pair canvas): readers recompute in-group values at xy offsets from the
+    staged inputs (1), also through recomputed values (2), or read shared-memory copies (0) --
+    the same IEEE operations in the same order, so the same bits as the oracle; on the weather
+    program (flux -> divergence chains, both periodic seams, ragged tiles) and on random programs."""
+    from .gpu_util import compare
+    for n in ((64, 48, 12), (40, 36, 10)):
+        desc = P.weather(n=n)
+        inputs = D.inputs_for(desc, 41)
+        ref = interp.run(desc, inputs, 2)
+        prog = kf.Program(desc)
+        tgt = kf.Target(tile=(32, 8, 0), pblock=(2, 1), inline_xy=level, minblocks=-1)
+        plan, _ = prog.search(kf.SEARCH_HGGA, tgt, seed=5)
+        got, _ = run_kf(desc, plan, inputs, 2, tgt)
+        assert compare(desc, got, ref) == [], (n, level)
+    for seed in range(4):
+        rng = np.random.default_rng(7000 + seed)
+        bc = tuple(int(x) for x in rng.integers(0, 2, size=3))
+        dtype = DT_F64 if seed % 2 else DT_F32
+        desc = P.random_program(7100 + seed, nk=6, na=4, n=(2 * int(rng.integers(8, 16)), 20, 8), dtype=dtype, bc=bc,
+                                max_r=1 + seed % 2)
+        inputs = D.uniform(desc, seed)
+        ref = interp.run(desc, inputs, 2)
+        for plan in sorted(En.legal_plans(desc), key=lambda p: len(set(p)))[:3]:
+            got, _ = run_kf(desc, plan, inputs, 2, kf.Target(tile=(16, 8, 0), pblock=(2, 1), inline_xy=level))
+            assert compare(desc, got, ref) == [], (seed, plan, level)
