@@ -1,7 +1,7 @@
 """One small fused run for compute-sanitizer (racecheck / synccheck / initcheck / memcheck).
 
   python tools/round2/sanitize_run.py tiny
-  python tools/round2/sanitize_run.py weather [pairs|points]
+  python tools/round2/sanitize_run.py weather [pairs|pairs_chunks|points]
 
 weather: 64x48x12 fp64 weather program, HGGA plan (seed 1), every group under the knobs the bench
 times (canvas pairs + pair z-queues + unpredicated canvas loads, or one point per thread), 2 steps,
@@ -35,6 +35,8 @@ def main():
         prog0 = kf.Program(desc)
         if mode == "pairs":
             tgt = kf.Target(tile=(32, 8, 0), pblock=(2, 1), pair_zq=1, canvas_ld=1, minblocks=-1)
+        elif mode == "pairs_chunks":   # z chunks of 5 planes: partial canvas iterations at chunk boundaries
+            tgt = kf.Target(tile=(32, 8, 5), pblock=(2, 1), pair_zq=1, canvas_ld=1, minblocks=-1)
         else:
             tgt = kf.Target(tile=(32, 8, 0), pblock=(1, 1), canvas_ld=1, minblocks=-1)
         plan, _ = prog0.search(kf.SEARCH_HGGA, tgt, seed=1)   # legal under this launch configuration (V8)
