@@ -232,14 +232,6 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
   std::set<int> canvas_pitches;
   for (auto& r : L.rings) canvas_pitches.insert(r.px);
   const bool pair_mode = canvas_mode && cv.pair;
-  // Partial canvas iterations (pair mode): stream iterations where some kernels are outside their
-  // plane range -- the pipeline fill / drain at an interior z-chunk boundary -- run the canvas too,
-  // every kernel computing (values of an inactive kernel are never stored nor read by an active
-  // one: a reader's planes lie in its producers' ranges) and ring stores guarded by the kernel's
-  // activity; only iterations with frozen ghost planes of an in-group producer (the domain's top
-  // and bottom, stored ghosts read from global memory, R9) keep the per-kernel slow path.  Carried
-  // z-queue values are reloaded after a partial iteration.
-  const bool partial = pair_mode && !getenv("KF_NO_PARTIAL");
   const int PSH = 2 * cv.lop - clo[0];   // pair mode: canvas x of the thread's first point = 2 * pair column - PSH
   // Clamped canvas loads (canvas_ld): a lane outside the reading kernels' regions never stores (nor
   // forwards to a stored point) what it computes, so it may load any address -- it loads the one of
@@ -925,8 +917,7 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
         const Kernel& K = p.kernels[k];
         const Ext& e = L.ext.at(k);
         const int ox = clo[0] - e.elo[0], oy = clo[1] - e.elo[1];
-        const std::string act = partial ? "act" + std::to_string(k) + " && " : "";
-        const std::string c0 = act + "ce" + std::to_string(k) + "_0", c1 = act + "ce" + std::to_string(k) + "_1";
+        const std::string c0 = "ce" + std::to_string(k) + "_0", c1 = "ce" + std::to_string(k) + "_1";
         bool any_out = false;
         for (size_t si = 0; si < K.stmts.size(); si++) {
           const Ver v{K.stmts[si].out, p.vw(k, K.stmts[si].out)};
@@ -965,7 +956,7 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
       else val = ldfirst_p.at(src.src);
       o << "      " << pq_name(pk) << " = " << val << ";\n";
     }
-    if (!pcarry.empty()) o << (partial ? "      pqv = t >= cf0 && t < cf1;\n" : "      pqv = true;\n");
+    if (!pcarry.empty()) o << "      pqv = true;\n";
   };
   auto qname = [](int k, const std::string& ps, int ring, int dz) {
     return "q" + std::to_string(k) + ps + "_" + std::to_string(ring) + "_" + (dz < 0 ? "m" + std::to_string(-dz) : std::to_string(dz));
@@ -1427,22 +1418,7 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
                    std::to_string(WY) + " <= NY";
     }
     if (!getenv("KF_CANVAS_COND")) c = "t >= cf0 && t < cf1";   // A/B switch: the per-kernel conjunction
-    if (partial) {
-      // no kernel on a ghost plane: p = t - delay outside [glo, plo) and [phi, ghi)
-      std::string gh;
-      for (int k : alive) {
-        const std::string ks = std::to_string(k), pz = "(t - " + std::to_string(L.delay.at(k)) + ")";
-        gh += std::string(gh.empty() ? "" : " || ") + "(" + pz + " >= glo" + ks + " && " + pz + " < plo" + ks + ") || (" + pz +
-              " >= phi" + ks + " && " + pz + " < ghi" + ks + ")";
-      }
-      c = "(t >= cf0 && t < cf1) || (cfxy && !(" + gh + "))";
-    }
     o << "    if (" << c << ") {   // ---- fast iteration on the canvas\n";
-    if (partial)
-      for (int k : alive) {
-        const std::string ks = std::to_string(k), pz = "(t - " + std::to_string(L.delay.at(k)) + ")";
-        o << "      const bool act" << ks << " = " << pz << " >= plo" << ks << " && " << pz << " < phi" << ks << ";\n";
-      }
     // clamped load bases (canvas_ld), recomputed every iteration from an opaque zero so the compiler
     // does not keep them live across the stream loop (cheap integer ops instead of registers)
     o << "      int kz;\n      asm volatile(\"mov.u32 %0, 0;\" : \"=r\"(kz));\n/*@@KF_CLAMP_BASES@@*/";
