@@ -5,6 +5,7 @@
 // traffic the generated kernel actually issues.
 #include <algorithm>
 #include <functional>
+#include <set>
 
 #include "kf_internal.hpp"
 
@@ -84,8 +85,11 @@ CanvasPlan plan_canvas(const Program& p, const GroupLowering& L) {
           const Ver V{K.stmts[si].out, p.vw(k, K.stmts[si].out)};
           if (L.ring_of(V) < 0 || c.inl.count(V)) continue;
           bool ok = true, any_xy = false;
+          int nloads = 0;
+          std::set<std::pair<int, int>> xy_offs;   // distinct nonzero xy offsets it is read at
           for (const Insn& in : K.stmts[si].rpn)
             if (in.op == KF_OP_LOAD) {
+              nloads++;
               const Ver W{in.arg, p.vr(k, in.arg)};
               const int r = L.ring_of(W);
               if (r < 0 || !(L.rings[r].live_in || c.inl.count(W))) ok = false;
@@ -96,10 +100,16 @@ CanvasPlan plan_canvas(const Program& p, const GroupLowering& L) {
             if (L.delay.at(c2) != L.delay.at(k)) ok = false;
             for (auto& d : it->second) {
               if (d[2] != 0) ok = false;
-              if (d[0] != 0 || d[1] != 0) any_xy = true;
+              if (d[0] != 0 || d[1] != 0) {
+                any_xy = true;
+                xy_offs.insert({d[0], d[1]});
+              }
             }
           }
           (void)any_xy;   // (values read only at offset 0 join too: the inputs of level-1 values)
+          // cost bound: a cheap producer read at few offsets (a flux read at i-1: 1 offset x 5
+          // loads); a wide stencil of a wide stencil (S13 of S27: 12 x 27) stays in shared memory
+          if (int(xy_offs.size()) * nloads > 16) ok = false;
           if (ok) add[V] = {k, int(si)};
         }
       }
