@@ -705,8 +705,13 @@ Codegen generate_group_kernel(const Program& p, const GroupLowering& L, int gid)
         const int off0 = (R.blo[1] - clo[1]) * R.px + (R.ax_lo - clo[0]);
         const int pk_ = R.producer;
         if (mod2(PSH + off0) != 0 || rel != off0 || po + 1 != -L.delay.at(pk_)) continue;
+        // Valid wherever it is used: a reader uses element j of the pair only at a point of its
+        // region, which lies in the producer's region (E(producer) covers its readers' regions
+        // grown by their offsets, here (0, 0)), where the previous fast iteration computed it.
+        // (Round 1 also required the key's lane rectangle -- widened by the pair's second element --
+        // inside the producer's rectangle, which rejected the z-flux carries.)
         const Rect rp = canvas_rect(L, cv, pk_);   // the producer's region (first point's x, both points inside)
-        if (rp[0] <= rc[0] && rp[1] - 1 >= rc[1] && rp[2] <= rc[2] && rp[3] >= rc[3])
+        if ((rp[0] <= rc[0] && rp[1] - 1 >= rc[1] && rp[2] <= rc[2] && rp[3] >= rc[3]) || !getenv("KF_OWN_CARRY_RECT"))
           pcarry[pk] = PSrc{false, nx, R.ver.x, R.ver.v};
       }
   }
