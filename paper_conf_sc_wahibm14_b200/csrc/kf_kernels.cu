@@ -114,10 +114,10 @@ __global__ void fill_xy_multi(FillList L, Geom g, int px, int py, int frozen_onl
 // Pieces: x spans of every row (x periodic; interior rows only if y is periodic as well), then
 // whole y-ghost rows (y periodic).  frozen_only (bits x/y/z frozen): only cells inside a frozen
 // axis' ghost layer, exact cells (the run-start fill of scratch buffers).
-template <typename T, int SEC>
+template <typename T>
 __global__ void fill_xy_sectors(FillList L, Geom g, int px, int py, int frozen_only) {
   T* base = (T*)L.base[blockIdx.y];
-  constexpr int E = SEC / sizeof(T);
+  constexpr int E = 32 / sizeof(T);
   const int NZ = g.nz + 2 * g.gz;
   const int xl0 = -((g.gx + E - 1) / E) * E;                 // left span [xl0, 0)
   const int xr0 = (g.nx / E) * E, xr1 = ((g.nx + g.gx + E - 1) / E) * E;   // right span [xr0, xr1)
@@ -242,12 +242,9 @@ cudaError_t launch_fill_xy_multi(void* const* bufs, int n, int px, int py, int e
   if (!px && !py) return cudaSuccess;
   const long long NZ = g.nz + 2 * g.gz;
   // sector-wide writes need the row origin (x = 0) 32-byte aligned (kf_array_layout: 128-byte rows)
-  // span granule: 32-byte sectors, or 64 bytes (KF_FILL_SPAN=64: whole DRAM bursts, A/B)
-  const int SEC = getenv("KF_FILL_SPAN") && atoi(getenv("KF_FILL_SPAN")) == 64 ? 64 : 32;
-  const int E = SEC / es;
-  const bool sectors = !getenv("KF_FILL_CELLS") && (g.xoff * (long long)es) % SEC == 0 && (g.pitch * (long long)es) % SEC == 0 &&
-                       (g.plane * (long long)es) % SEC == 0 && ((g.gx + E - 1) / E) * E <= g.xoff &&
-                       ((g.nx + g.gx + E - 1) / E) * E <= g.pitch - g.xoff;
+  const int E = 32 / es;
+  const bool sectors = !getenv("KF_FILL_CELLS") && (g.xoff * (long long)es) % 32 == 0 && (g.pitch * (long long)es) % 32 == 0 &&
+                       (g.plane * (long long)es) % 32 == 0 && ((g.gx + E - 1) / E) * E <= g.xoff;
   long long per = (px ? 2LL * g.gx * (g.ny + 2 * g.gy) : 0) * NZ +
                   (py ? (long long)(px ? g.nx : g.nx + 2 * g.gx) * 2 * g.gy * NZ : 0);
   if (sectors) {
@@ -263,10 +260,8 @@ cudaError_t launch_fill_xy_multi(void* const* bufs, int n, int px, int py, int e
     long long nb = (per + 255) / 256;
     const long long cap = (148LL * 16 + m - 1) / m;   // ~16 CTAs per SM over all buffers
     dim3 grid(unsigned(nb < cap ? nb : cap), unsigned(m));
-    if (sectors && SEC == 64 && es == 4) fill_xy_sectors<float, 64><<<grid, 256, 0, s>>>(L, g, px, py, frozen_only);
-    else if (sectors && SEC == 64) fill_xy_sectors<double, 64><<<grid, 256, 0, s>>>(L, g, px, py, frozen_only);
-    else if (sectors && es == 4) fill_xy_sectors<float, 32><<<grid, 256, 0, s>>>(L, g, px, py, frozen_only);
-    else if (sectors) fill_xy_sectors<double, 32><<<grid, 256, 0, s>>>(L, g, px, py, frozen_only);
+    if (sectors && es == 4) fill_xy_sectors<float><<<grid, 256, 0, s>>>(L, g, px, py, frozen_only);
+    else if (sectors) fill_xy_sectors<double><<<grid, 256, 0, s>>>(L, g, px, py, frozen_only);
     else if (es == 4) fill_xy_multi<float><<<grid, 256, 0, s>>>(L, g, px, py, frozen_only);
     else fill_xy_multi<double><<<grid, 256, 0, s>>>(L, g, px, py, frozen_only);
   }
