@@ -851,7 +851,7 @@ def run_kf(args):
                                    f"overlapped with interior tiles, CUDA graph), {wl.scaling}") if world > 1 else "1 GPU",
                    "local_grid": list(desc.n), "global_points": wl.global_npts,
                    "graph": True, "jit_s": round(jit_s, 2),
-                   "per_group_launch_config": tuned if tuned else "uniform",
+                   "per_group_launch_config": [cand_norm(c) for c in tuned] if tuned else "uniform",
                    "plan_candidates": candidates,
                    "autotune_tried": [{"config": list(c), "group_ms": [round(x, 4) for x in g]} for c, g in tried]
                    if tried else None},
