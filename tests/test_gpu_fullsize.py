@@ -64,8 +64,8 @@ def test_weather_full_size_bench_configuration():
     desc = P.weather(n=(512, 512, 128))
     inputs = D.weather_inputs(desc, 3)
     prog = kf.Program(desc)
-    gt = [kf.Target(tile=tuple(c[0]), stages=c[1], zunroll=c[2], ringunroll=c[3], minblocks=c[4], canvas_ld=c[5],
-                    pblock=(c[6], 1), pair_zq=c[7], ghostwrite=gw) for c in tuned]
+    import bench
+    gt = [kf.Target(**dict(bench.cand_kw({}, c), ghostwrite=gw)) for c in tuned]
     nsteps = 2
     ex = kf.Exec(prog, plan, kf.Target(tile=(32, 8, 64)), group_targets=gt)
     if gw:
